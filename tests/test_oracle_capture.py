@@ -1,0 +1,86 @@
+"""Whole-path oracle invariants (BASELINE.json north_star):
+restore(capture(S)) == S bitwise, the union of shards covers every byte once,
+identical replicas give equal digests, a flip in the committed image is caught
+at the exact chunk, and an uncommitted checkpoint is refused (PAPER.md:136,
+:140)."""
+import numpy as np
+
+from oracle import oracle as O
+from workloads import configs as W
+
+
+def _c1_small():
+    return W.scaled(W.c1(), 3000)
+
+
+def test_identical_replicas_equal_digests_and_roundtrip():
+    w = _c1_small()
+    g = w.groups[0]
+    lay = O.layout_of_group(g, 4096)
+    imgs, ds = {}, {}
+    for r in range(2):               # two DP replicas generated from the same seed
+        imgs[r] = O.pack(O.gen_group(g, w.seed), lay)
+        ds[r] = O.jf64(imgs[r], lay.C, 0, lay.n_c)
+    assert np.array_equal(ds[0], ds[1])
+    for k in (1, 2):
+        gs = O.GroupSel(0, O.REQUIRED, writers=list(range(k)))
+        st, host, man, com = O.capture_sim(gs, 3, lay, imgs, ds)
+        assert st == O.OK and np.array_equal(host, imgs[0])
+        st, bad, ts = O.restore_sim(host, man, com)
+        assert st == O.OK
+        for a, b in zip(ts, O.gen_group(g, w.seed)):
+            assert np.array_equal(a, b)
+
+
+def test_corrupt_image_exact_chunk():
+    w = _c1_small()
+    g = w.groups[0]
+    lay = O.layout_of_group(g, 4096)
+    img = O.pack(O.gen_group(g, w.seed), lay)
+    d = O.jf64(img, lay.C, 0, lay.n_c)
+    gs = O.GroupSel(0, O.REQUIRED, writers=[0])
+    st, host, man, com = O.capture_sim(gs, 3, lay, {0: img}, {0: d})
+    rng = np.random.default_rng(0)
+    for _ in range(20):
+        pos = int(rng.integers(0, lay.L))
+        h = host.copy(); h[pos] ^= 1 << int(rng.integers(0, 8))
+        st, bad, _ = O.restore_sim(h, man, com)
+        assert st == O.ECORRUPT and bad == pos // lay.C
+
+
+def test_uncommitted_refused():
+    w = _c1_small()
+    g = w.groups[0]
+    lay = O.layout_of_group(g, 4096)
+    img = O.pack(O.gen_group(g, w.seed), lay)
+    d = O.jf64(img, lay.C, 0, lay.n_c)
+    gs = O.GroupSel(0, O.REQUIRED, writers=[0])
+    _, host, man, com = O.capture_sim(gs, 3, lay, {0: img}, {0: d})
+    assert O.restore_sim(host, man, None)[0] == O.EINCOMPLETE
+    assert O.restore_sim(host, None, com)[0] == O.EINCOMPLETE
+    bad = bytearray(man); bad[100] ^= 1            # a torn / altered manifest
+    assert O.restore_sim(host, bytes(bad), com)[0] == O.EINCOMPLETE
+
+
+def test_half_step_detected():
+    """A half-applied optimizer step (U_v on tensors [0, split)) changes the
+    digests of exactly the chunks those tensors touch."""
+    w = _c1_small()
+    g = w.groups[0]
+    lay = O.layout_of_group(g, 4096)
+    ts = O.gen_group(g, w.seed)
+    d0 = O.jf64(O.pack(ts, lay), lay.C, 0, lay.n_c)
+    L = O.lib()
+    for split in range(1, len(ts), 17):
+        t2 = [t.copy() for t in ts]
+        for i in range(split):
+            if g.tensors[i].dtype == "f32":
+                x = t2[i].view(np.uint32)
+                L.orc_update_fp32(O._ptr(x), 0, len(x), g.tensors[i].gen_id, 4)
+        d1 = O.jf64(O.pack(t2, lay), lay.C, 0, lay.n_c)
+        touched = set()
+        for i in range(split):
+            touched |= set(range(lay.offsets[i] // lay.C, (lay.offsets[i] + lay.nbytes[i] - 1) // lay.C + 1))
+        changed = set(np.nonzero(d0 != d1)[0].tolist())
+        assert changed == touched
+        assert O.root(lay.layout_hash, d0) != O.root(lay.layout_hash, d1)
