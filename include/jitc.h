@@ -1,0 +1,280 @@
+/*
+ * jitc.h -- C ABI of the B200-native just-in-time checkpoint capture/restore
+ * library (libjitc.so).  Hot path of "Just-In-Time Checkpointing: Low Cost
+ * Error Recovery from Deep Learning Training Failures" (Gupta et al.,
+ * EuroSys '24); paper text at PAPER.md, cited as PAPER.md:<line> (§section).
+ *
+ * The paper's user-level library takes a user `save_checkpoint` callback and
+ * returns a replica checkpoint path (PAPER.md:99 §3, :132 §3.2, :140 §3.3).
+ * This ABI replaces both with explicit calls on the GPU state of healthy
+ * data-parallel replicas:
+ *
+ *   register (steady state) -> mark (every optimizer step)
+ *   on failure: fingerprint -> exchange_records -> select_consistent_replica
+ *               -> capture (shard s of k) -> commit
+ *   on restart / replacement: restore -> verify
+ *
+ * Conventions (all functions):
+ *  - Every call returns a jitc_status; 0 == JITC_OK.  On error, the text of
+ *    jitc_last_error(ctx) (or jitc_last_error(NULL) for ctx-less calls,
+ *    thread-local) says why.  No call aborts the process.
+ *  - Pointers: "device" = CUDA device memory of cfg.device (e.g. torch
+ *    tensors' data_ptr); "host" = ordinary host memory.  Tensor pointers,
+ *    staging and streams are CALLER-OWNED and must stay valid and unmoved
+ *    until jitc_destroy or a re-register; the library never frees them.  Host
+ *    images, manifests, digests and events are LIBRARY-OWNED.
+ *  - Blocking: each call returns after its GPU work has completed.  It waits
+ *    only on the library's own non-blocking streams and events -- never on
+ *    the legacy default stream, never cudaDeviceSynchronize -- and
+ *    fingerprint / capture / restore / verify never allocate, free or pin
+ *    (all of that happens in create / register).  This generalises
+ *    PAPER.md:134 (copies re-issued on a new stream because the default
+ *    stream is blocked behind the hung collective).
+ *  - Threading: one thread per ctx at a time; callable from a non-Python
+ *    watchdog thread (no callbacks, so no GIL).
+ *  - Collective calls (every member of the library communicator must call):
+ *    jitc_comm_init, jitc_comm_shrink, jitc_exchange_records, jitc_commit,
+ *    jitc_restore.  Local: register, declare_group, mark, fingerprint,
+ *    capture, verify.  Pure (no ctx, no GPU): jitc_layout, jitc_shard_range,
+ *    jitc_select_consistent_replica.
+ *  - No CPU fallback: if the device or the sm_100a kernels are unavailable
+ *    the call fails with JITC_ECUDA.
+ *  - Binary formats (record blob, selection, manifest, commit record) are
+ *    little-endian and specified in DESIGN.md §Formats.
+ */
+#ifndef JITC_H_
+#define JITC_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define JITC_ABI_VERSION 1
+#define JITC_ALL_GROUPS 0xFFFFFFFFu
+
+typedef struct jitc_ctx jitc_ctx;
+typedef int32_t jitc_status;
+
+enum {
+    JITC_OK = 0,
+    JITC_EINVAL = -1,          /* bad argument                                          */
+    JITC_ESTATE = -2,          /* call out of order (e.g. capture before fingerprint)   */
+    JITC_ENOMEM = -3,          /* device / pinned host allocation failed                 */
+    JITC_ECUDA = -4,           /* CUDA runtime error (incl. no device / no sm_100a)      */
+    JITC_ENCCL = -5,           /* NCCL error                                             */
+    JITC_ELAYOUT = -6,         /* replicas registered different tensors / topology       */
+    JITC_ENOREPLICA = -7,      /* a REQUIRED group has no healthy replica */
+    JITC_ECONFLICT = -8,       /* tie between differing replica classes                  */
+    JITC_ENOCONSISTENT = -9,   /* no version common to all REQUIRED groups*/
+    JITC_EUNSTABLE = -10,      /* bytes changed between fingerprint and capture          */
+    JITC_ECORRUPT = -11,       /* restored bytes do not match the manifest digests       */
+    JITC_EINCOMPLETE = -12,    /* checkpoint not committed (PAPER.md:136 metadata last)  */
+    JITC_EIO = -13             /* file / shm error                                       */
+};
+
+/* Optimizer-step phase of a group, written by jitc_mark (PAPER.md:188 hooks). */
+enum { JITC_PHASE_CLEAN = 0, JITC_PHASE_DIRTY = 1 };
+/* Group policy: REQUIRED state must be recovered; OPTIONAL (grads-like) state
+ * is kept only if consistent at the selected version (reading R1). */
+enum { JITC_REQUIRED = 0, JITC_OPTIONAL = 1 };
+/* Restore source: HOST = the committed host image (every rank restarts,
+ * PAPER.md:116); PEER = the writers' live HBM over NVLink (only the
+ * replacement lost its state). */
+enum { JITC_RESTORE_HOST = 0, JITC_RESTORE_PEER = 1 };
+/* Per-group selection status (jitc_sel_group.status). */
+enum { JITC_G_OK = 0, JITC_G_UNVERIFIED_SINGLE = 1, JITC_G_NOREPLICA = 2, JITC_G_DROPPED = 3,
+       JITC_G_CONFLICT = 4, JITC_G_NOCANDIDATE = 5 };
+/* Reason a healthy member is not a writer (O6 step 10). */
+enum { JITC_X_DIRTY = 1, JITC_X_STALE_VERSION = 2, JITC_X_MINORITY = 3 };
+/* jitc_config.flags */
+enum {
+    JITC_F_ZERO_COPY_D2H = 1u << 0,  /* capture: K2 stores straight into mapped pinned host memory */
+    JITC_F_ZERO_COPY_H2D = 1u << 1,  /* restore: K3 loads straight from mapped pinned host memory  */
+    JITC_F_TIME_KERNELS = 1u << 2,   /* bracket every kernel launch with CUDA events (stats)        */
+    JITC_F_NO_SHM_UNLINK = 1u << 3   /* keep /dev/shm images after a verified restore               */
+};
+
+typedef struct {
+    int32_t device;          /* CUDA device ordinal                                          */
+    int32_t rank;            /* this process's job rank (member lists use job ranks)         */
+    int32_t world;           /* job world size                                               */
+    uint32_t flags;          /* JITC_F_*                                                     */
+    uint64_t chunk_bytes;    /* digest chunk C: power of two in [4 KiB, 64 MiB]; 0 => 1 MiB  */
+    void* staging;           /* device staging buffer (caller-owned) or NULL => library      */
+    uint64_t staging_bytes;  /* staging size; 0 => 1 GiB.  Split into rounds of slot_bytes.  */
+    uint64_t slot_bytes;     /* bytes per pipeline round (multiple of C); 0 => 256 MiB       */
+    const char* image_dir;   /* host image location: a directory on /dev/shm shared by the
+                                ranks of one box (survives process death), or NULL =>
+                                private pinned memory (writers must stay alive)               */
+    void* streams[2];        /* caller-created non-blocking cudaStream_t (compute, copy) or
+                                NULL => library-created                                       */
+} jitc_config;
+
+/* dtype is an opaque tag folded into layout_hash (the workloads use
+ * 0=u8, 1=bf16, 2=f32); the path itself moves bytes. */
+typedef struct {
+    const char* name;        /* stable name, identical on every replica   */
+    void* ptr;               /* device pointer; any alignment (16-B aligned is fastest)      */
+    uint64_t nbytes;         /* may be 0 and need not be a multiple of anything              */
+    uint32_t dtype;
+} jitc_tensor;
+
+/* Per-call statistics (optional out-parameter; may be NULL). */
+typedef struct {
+    double ms_host;            /* wall time of the call                                        */
+    double ms_device;          /* CUDA-event span of the call on the library streams           */
+    double ms_kernel;          /* sum of the call's kernel durations (needs JITC_F_TIME_KERNELS)*/
+    uint64_t image_bytes;      /* image bytes this rank packed / unpacked / digested           */
+    uint64_t d2h_bytes, h2d_bytes, p2p_bytes;
+    uint64_t kernel_launches;  /* launches of this library's kernels during the call           */
+    uint32_t rounds;           /* pipeline rounds                                              */
+    int32_t first_bad_chunk;   /* ECORRUPT: first chunk whose digest mismatched, else -1       */
+} jitc_stats;
+
+/* Cumulative per-kernel counters (bench roofline): kind 1 = K1 digest,
+ * 2 = K2 pack+digest, 3 = K3 unpack+verify. */
+typedef struct {
+    uint64_t launches;
+    uint64_t bytes;            /* algorithmic image bytes processed                            */
+    double ms;                 /* sum of CUDA-event launch durations (JITC_F_TIME_KERNELS)     */
+} jitc_kernel_counter;
+
+/* ---- lifecycle --------------------------------------------------------- */
+/* Creates a context on cfg->device: streams (unless given), events, staging
+ * (unless given).  Fails with JITC_ECUDA if the device is not sm_100. */
+jitc_status jitc_create(const jitc_config* cfg, jitc_ctx** out);
+void jitc_destroy(jitc_ctx* ctx);
+/* Thread-local text of the last error (ctx may be NULL). Never NULL. */
+const char* jitc_last_error(const jitc_ctx* ctx);
+int jitc_abi_version(void);
+
+/* ---- steady state ------------------------------------------------------ */
+/* A1: registers `n` tensors of `group` held by this rank and
+ * declares the group's policy and job-rank members (this rank must be one).
+ * Builds the image layout (registration order, 256-B aligned offsets, zero
+ * padding; reading R4), the segment table, per-group digest buffers, and
+ * maps/pins the host image (image_dir/g<group>.img, or private pinned).
+ * Out: layout_hash (fold of names, sizes, dtypes, C) and image_bytes (L). */
+jitc_status jitc_register(jitc_ctx* ctx, uint32_t group, int32_t policy, const int32_t* members,
+                          int32_t n_members, const jitc_tensor* t, size_t n, uint64_t* layout_hash,
+                          uint64_t* image_bytes);
+/* Declares a group this rank does NOT hold (e.g. another rank's ZeRO shard),
+ * so the selection can tell "no replica" from "not part of the job". */
+jitc_status jitc_declare_group(jitc_ctx* ctx, uint32_t group, int32_t policy, const int32_t* members,
+                               int32_t n_members);
+/* A2: stream-ordered phase word of `group`: version<<1 | phase, one atomic
+ * 8-B write into mapped pinned host memory, issued with cuStreamWriteValue64
+ * on `stream` (after the optimizer kernels already queued there; no kernel,
+ * no sync).  stream == NULL writes immediately from the host.  Mirrors the
+ * pre/post-optimizer-step hooks of PAPER.md:188. */
+jitc_status jitc_mark(jitc_ctx* ctx, uint32_t group, uint64_t version, int32_t phase, void* stream);
+/* Reads the phase word as the capture will see it. */
+jitc_status jitc_phase(jitc_ctx* ctx, uint32_t group, uint64_t* version, int32_t* phase);
+
+/* ---- communicator (NCCL over NVLink/NVSwitch) ---------------------------- */
+/* 128-byte ncclUniqueId (rank 0 creates, the harness distributes it). */
+jitc_status jitc_get_unique_id(void* id128);
+/* Library-owned NCCL communicator of `nranks`; comm rank i <-> job rank
+ * job_ranks[i] (NULL => identity). */
+jitc_status jitc_comm_init(jitc_ctx* ctx, const void* id128, int32_t nranks, int32_t comm_rank,
+                           const int32_t* job_ranks);
+/* Drops `failed` job ranks with ncclCommShrink(NCCL_SHRINK_ABORT), which also
+ * aborts collectives hung on the old communicator (PAPER.md:180 re-establish
+ * comms; Table 7 shows this dominates recovery). */
+jitc_status jitc_comm_shrink(jitc_ctx* ctx, const int32_t* failed, int32_t n_failed);
+jitc_status jitc_comm_destroy(jitc_ctx* ctx);
+
+/* ---- on failure: capture --------------------------------------------------- */
+/* A3 = K1: JF64 chunk digests of every registered byte of `group` (or all
+ * held groups with JITC_ALL_GROUPS), read from live HBM, plus the phase word.
+ * Output: this rank's record blob (header, topology, one record per group;
+ * DESIGN.md §Formats).  cap == 0 => only *len (the needed size) is set.
+ * The checksum primitive the paper uses for replay validation,
+ * here the replica-consistency evidence. */
+jitc_status jitc_fingerprint(jitc_ctx* ctx, uint32_t group, void* blob, size_t cap, size_t* len);
+/* A4 = C1: all-gathers every member's blob over the library communicator
+ * (blob sizes first, then the padded blobs) and writes them, compacted and
+ * in comm-rank order, to `all`.  Without a communicator (single process)
+ * copies `mine`.  cap == 0 => only *all_len. */
+jitc_status jitc_exchange_records(jitc_ctx* ctx, const void* mine, size_t len, void* all, size_t cap,
+                                  size_t* all_len);
+/* A5 (pure): the consistency rule O6.  Keeps blobs of
+ * `healthy` job ranks; per group the unique largest class of identical CLEAN
+ * records per version; v* = max version at which every REQUIRED group has a
+ * candidate; writers = that class; the rest excluded
+ * with a reason.  Returns the overall status (also stored in the selection);
+ * the selection is written even on ELAYOUT/ENOREPLICA/ECONFLICT/
+ * ENOCONSISTENT for diagnostics.  Every rank computes the same bytes. */
+jitc_status jitc_select_consistent_replica(const void* blobs, size_t len, const int32_t* healthy,
+                                           int32_t n_healthy, void* selection, size_t cap,
+                                           size_t* sel_len);
+/* A6+A7 = K2 + D2H: if this rank is writer s of k for `group` (or for each
+ * held group with JITC_ALL_GROUPS) it packs its chunk range
+ * [floor(s*n_c/k), floor((s+1)*n_c/k)) (O5) into the host image, in rounds:
+ * K2 gathers the tensors into a staging slot (or straight into mapped host
+ * memory with JITC_F_ZERO_COPY_D2H) re-digesting every chunk, and the copy
+ * stream drains the slot D2H while K2 fills the next.  A re-digest that
+ * differs from the last jitc_fingerprint => JITC_EUNSTABLE.  A non-writer
+ * returns JITC_OK having done nothing, so every rank can call it. */
+jitc_status jitc_capture(jitc_ctx* ctx, const void* selection, size_t sel_len, uint32_t group,
+                         jitc_stats* stats);
+/* A8: after every writer's capture, writes per group the manifest (header,
+ * tensor table, digests, root, shard map, v*) and LAST the commit record
+ * ("metadata file is stored at the end").  Collective: a
+ * barrier on the communicator orders "all shards done" before the manifest;
+ * the lowest-rank writer of each group writes it. */
+jitc_status jitc_commit(jitc_ctx* ctx, const void* selection, size_t sel_len);
+
+/* ---- restore ------------------------------------------------------------- */
+/* A9-A11.  HOST: refuses an uncommitted image (JITC_EINCOMPLETE); each comm
+ * rank loads chunk range O5(n_c, n, r) H2D, the ranks all-gather the slices
+ * over NVLink in rounds, and K3 scatters every round into the registered
+ * tensors while re-digesting it; any chunk whose digest differs from the
+ * manifest => JITC_ECORRUPT (stats->first_bad_chunk).  PEER: the selection's
+ * writers pack their ranges from live HBM (K2) and send them to every member
+ * that is not a writer (the replacement, and members excluded as DIRTY /
+ * MINORITY / STALE), which unpack+verify with K3 against the writers'
+ * digests.  selection may be NULL in HOST mode (taken from the manifest). */
+jitc_status jitc_restore(jitc_ctx* ctx, uint32_t group, int32_t mode, const void* selection,
+                         size_t sel_len, jitc_stats* stats);
+/* A12: K1 over the live tensors of `group`, compared with `expected` (a
+ * record blob holding that group) or, if NULL, with the manifest digests of
+ * the last restore / commit.  Mismatch => JITC_ECORRUPT, *first_bad_chunk
+ * set (else UINT64_MAX). */
+jitc_status jitc_verify(jitc_ctx* ctx, uint32_t group, const void* expected, size_t len,
+                        uint64_t* first_bad_chunk);
+
+/* ---- pure helpers --------------------------------------------------------- */
+/* O1 layout: offsets (may be NULL; n entries), layout_hash, image_bytes. */
+jitc_status jitc_layout(const jitc_tensor* t, size_t n, uint64_t chunk_bytes, uint64_t* offsets,
+                        uint64_t* layout_hash, uint64_t* image_bytes);
+/* O5 shard rule: writer s of k gets chunks [*c0, *c1). */
+jitc_status jitc_shard_range(uint64_t n_c, uint32_t k, uint32_t s, uint64_t* c0, uint64_t* c1);
+
+/* ---- counters ---------------------------------------------------------------- */
+jitc_status jitc_kernel_counters(jitc_ctx* ctx, int32_t kind, jitc_kernel_counter* out);
+jitc_status jitc_reset_counters(jitc_ctx* ctx);
+
+/* ---- test/bench harness kernels (K4; not part of the method) ------------- */
+/* Fills numel elements of a device tensor with the O9 counter-based generator
+ * (dtype 0=u8,1=bf16,2=f32,3=zeros,4=ones).  Integer-only, so bit-identical
+ * with the oracle's generator. */
+jitc_status jitc_gen_fill(void* dptr, uint32_t dtype, uint64_t numel, uint64_t seed, uint32_t group,
+                          uint32_t gen_id, uint32_t exp_lo, uint32_t exp_hi, int32_t force_pos,
+                          void* stream);
+/* O10 synthetic optimizer update U_v on elements [e0, e0+count) of the fp32
+ * device tensor whose element 0 is at dptr; and bf16 params re-derived as
+ * RNE(master). */
+jitc_status jitc_inject_update(void* dptr, uint64_t e0, uint64_t count, uint32_t gen_id, uint64_t v,
+                               void* stream);
+jitc_status jitc_inject_rne(const void* master_f32, void* param_bf16, uint64_t count, void* stream);
+/* Flips bit `bit` of byte `byte` of device memory at dptr. */
+jitc_status jitc_inject_bitflip(void* dptr, uint64_t byte, uint32_t bit, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* JITC_H_ */

@@ -1,0 +1,333 @@
+// sm_100a kernels of libjitc.so.
+//
+//  K1 digest        : JF64 chunk digests of live tensors (reads L from HBM)
+//  K2 pack+digest   : gather tensors -> contiguous image bytes (staging slot in
+//                     HBM, or mapped pinned host memory), JF64 in the same pass
+//  K3 unpack+verify : image bytes (staging slot / mapped host) -> scatter into
+//                     the tensors, JF64 of the bytes read
+//  K4 (harness)     : counter-based synthetic state, optimizer-update and
+//                     bit-flip injectors
+//
+// JF64 (reading R2; PAPER.md:162 names only "checksums"): for image word g
+// (8 bytes, little-endian) term(g) = fmix64(w ^ (g+1)*PHI); d[chunk] is the
+// wrap-around sum of its terms.  The sum is order-free, so every CTA adds its
+// partial into d[chunk] with a 64-bit atomic and the result is deterministic.
+//
+// Work unit: one Seg = one piece (<= 128 KiB) of one tensor that never crosses
+// a chunk boundary.  A persistent grid of CTAs strides over segments; inside
+// a segment every thread streams 16-byte vectors (4 loads in flight before
+// any use), hashes both words, optionally stores, and the warp reduces its
+// partial with shuffles before one atomicAdd per warp per segment.  Pure HBM
+// (or PCIe) streaming: no tensor cores, no shared-memory reuse (every byte is
+// touched once), so the design targets coalescing, MLP and a grid sized to
+// the SM count.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "jitc_internal.h"
+
+namespace jitc {
+
+namespace {
+
+constexpr int kThreads = 256;
+constexpr int kUnroll = 4;
+constexpr uint64_t PHI = 0x9E3779B97F4A7C15ull;
+
+__device__ __forceinline__ uint64_t dmix(uint64_t x) {
+  x ^= x >> 33;
+  x *= 0xff51afd7ed558ccdull;
+  x ^= x >> 33;
+  x *= 0xc4ceb9fe1a85ec53ull;
+  x ^= x >> 33;
+  return x;
+}
+
+__device__ __forceinline__ uint4 ld_stream(const uint4* p) {
+  uint4 v;
+  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint4 ld_plain(const uint4* p) { return __ldcs(p); }
+__device__ __forceinline__ void st_stream(uint4* p, uint4 v) { __stcs(p, v); }
+__device__ __forceinline__ uint64_t lo64(uint4 v) { return (uint64_t)v.x | ((uint64_t)v.y << 32); }
+__device__ __forceinline__ uint64_t hi64(uint4 v) { return (uint64_t)v.z | ((uint64_t)v.w << 32); }
+
+// Assemble the little-endian word made of bytes [b, b+8) of a tensor piece
+// whose first `data` bytes come from `src` (any alignment) and the rest are 0.
+__device__ __forceinline__ uint64_t load_word_bytes(const uint8_t* src, uint64_t b, uint64_t data,
+                                                    bool al8) {
+  if (al8 && b + 8 <= data) return *reinterpret_cast<const uint64_t*>(src + b);
+  uint64_t w = 0;
+#pragma unroll
+  for (int i = 7; i >= 0; --i) {
+    uint64_t bi = b + i;
+    uint64_t byte = bi < data ? (uint64_t)src[bi] : 0ull;
+    w = (w << 8) | byte;
+  }
+  return w;
+}
+
+__device__ __forceinline__ void store_word_bytes(uint8_t* dst, uint64_t b, uint64_t data, uint64_t w,
+                                                 bool al8) {
+  if (al8 && b + 8 <= data) {
+    *reinterpret_cast<uint64_t*>(dst + b) = w;
+    return;
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+    if (b + i < data) dst[b + i] = (uint8_t)(w >> (8 * i));
+}
+
+__device__ __forceinline__ uint64_t warp_sum(uint64_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ segs, LaunchRanges R,
+                                                       unsigned long long* __restrict__ dig) {
+  const uint32_t total = R.prefix[R.n];
+  const int tid = threadIdx.x;
+  const int lane = tid & 31;
+  for (uint32_t v = blockIdx.x; v < total; v += gridDim.x) {
+    int r = 0;
+    while (v >= R.prefix[r + 1]) ++r;
+    const Seg sg = segs[R.seg_begin[r] + (v - R.prefix[r])];
+    const uint64_t rel = sg.img_off - R.base_off[r];
+    uint8_t* img = reinterpret_cast<uint8_t*>(R.base[r]) + rel;  // 16-B aligned (staging / host image)
+    uint8_t* ten = reinterpret_cast<uint8_t*>(sg.src);
+    const uint64_t data = sg.data_bytes;
+    const uint64_t words = (data + sg.pad_bytes) >> 3;
+    const uint64_t g0 = sg.img_off >> 3;
+    uint64_t acc = 0;
+    uint64_t body_words = 0;
+
+    if (sg.flags & kSegAligned16) {
+      const uint32_t nvec = (uint32_t)(data >> 4);
+      body_words = 2ull * nvec;
+      const uint4* in = MODE == kUnpack ? reinterpret_cast<const uint4*>(img)
+                                        : reinterpret_cast<const uint4*>(ten);
+      uint4* out = MODE == kPack ? reinterpret_cast<uint4*>(img)
+                 : MODE == kUnpack ? reinterpret_cast<uint4*>(ten) : nullptr;
+      uint32_t i = tid;
+      // key of word 2i is (g0 + 2i + 1) * PHI; the step between a thread's
+      // consecutive vectors is 2 * kThreads words.
+      uint64_t key = (g0 + 2ull * i + 1ull) * PHI;
+      const uint64_t kstep = 2ull * kThreads * PHI;
+      for (; i + (kUnroll - 1) * kThreads < nvec; i += kUnroll * kThreads) {
+        uint4 x[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) x[u] = MODE == kUnpack ? ld_plain(in + i + u * kThreads)
+                                                                 : ld_stream(in + i + u * kThreads);
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+          acc += dmix(lo64(x[u]) ^ key);
+          acc += dmix(hi64(x[u]) ^ (key + PHI));
+          key += kstep;
+          if (MODE != kDigest) st_stream(out + i + u * kThreads, x[u]);
+        }
+      }
+      for (; i < nvec; i += kThreads) {
+        uint4 x = MODE == kUnpack ? ld_plain(in + i) : ld_stream(in + i);
+        acc += dmix(lo64(x) ^ key);
+        acc += dmix(hi64(x) ^ (key + PHI));
+        key += kstep;
+        if (MODE != kDigest) st_stream(out + i, x);
+      }
+    }
+    // Remaining words: unaligned tensors (all of them), the < 16-byte data
+    // tail, and the zero padding that closes the tensor's image slot.
+    const bool al8 = (sg.flags & kSegAligned8) != 0;
+    for (uint64_t w = body_words + tid; w < words; w += kThreads) {
+      const uint64_t b = 8 * w;
+      uint64_t x;
+      if (MODE == kUnpack) {
+        x = *reinterpret_cast<const uint64_t*>(img + b);
+        if (b < data) store_word_bytes(ten, b, data, x, al8);
+      } else {
+        x = load_word_bytes(ten, b, data, al8);
+        if (MODE == kPack) *reinterpret_cast<uint64_t*>(img + b) = x;
+      }
+      acc += dmix(x ^ ((g0 + w + 1ull) * PHI));
+    }
+    acc = warp_sum(acc);
+    if (lane == 0) atomicAdd(dig + sg.chunk, (unsigned long long)acc);
+  }
+}
+
+__global__ void phase_write_kernel(volatile uint64_t* slot, uint64_t value) {
+  *slot = value;
+  __threadfence_system();
+}
+
+// ----------------------------------------------------------------- K4 (harness)
+__device__ __forceinline__ uint64_t dsplitmix(uint64_t z) {
+  z += PHI;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+__device__ __forceinline__ uint32_t gen_bits(uint64_t key, uint64_t seed, uint64_t j, uint32_t lo,
+                                             uint32_t span, int pos) {
+  uint64_t x = dsplitmix(seed ^ key ^ j);
+  uint32_t sign = pos ? 0u : (uint32_t)(x >> 63);
+  uint32_t e = lo + (uint32_t)(((x >> 32) & 0xFFFFull) % span);
+  return (sign << 31) | (e << 23) | (uint32_t)(x & 0x7FFFFFull);
+}
+__device__ __forceinline__ uint16_t to_bf16_rne(uint32_t u) {
+  return (uint16_t)((u + 0x7FFFu + ((u >> 16) & 1u)) >> 16);
+}
+
+__global__ void gen_kernel(uint8_t* out, uint32_t dtype, uint64_t numel, uint64_t seed, uint64_t key,
+                           uint32_t lo, uint32_t span, int pos) {
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < numel; j += stride) {
+    switch (dtype) {
+      case 0: {  // u8: byte b = byte (b % 4) of fp32 word (b / 4)
+        uint32_t w = gen_bits(key, seed, j >> 2, lo, span, pos);
+        out[j] = (uint8_t)(w >> (8 * (j & 3)));
+        break;
+      }
+      case 1:
+        reinterpret_cast<uint16_t*>(out)[j] = to_bf16_rne(gen_bits(key, seed, j, lo, span, pos));
+        break;
+      case 2:
+        reinterpret_cast<uint32_t*>(out)[j] = gen_bits(key, seed, j, lo, span, pos);
+        break;
+      case 3:
+        out[j] = 0;
+        break;
+      default:
+        out[j] = 0xFF;
+        break;
+    }
+  }
+}
+
+__global__ void update_kernel(uint32_t* x, uint64_t e0, uint64_t count, uint64_t tid_key, uint64_t vkey) {
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += stride) {
+    uint64_t j = e0 + i;
+    uint64_t h = dmix((tid_key ^ j) ^ vkey);
+    x[j] ^= (uint32_t)(h & 0xFFFFull);
+  }
+}
+
+__global__ void rne_kernel(const uint32_t* m, uint16_t* p, uint64_t count) {
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += stride)
+    p[i] = to_bf16_rne(m[i]);
+}
+
+__global__ void bitflip_kernel(uint8_t* p, uint8_t mask) { *p ^= mask; }
+
+int g_grid[64] = {0};
+
+}  // namespace
+
+int segment_grid(int device) {
+  if (device < 0 || device >= 64) return 148 * 8;
+  if (!g_grid[device]) {
+    int sms = 148, per = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, seg_kernel<kPack>, kThreads, 0);
+    if (per <= 0) per = 4;
+    g_grid[device] = sms * per;
+  }
+  return g_grid[device];
+}
+
+cudaError_t device_check(int device, std::string* why) {
+  cudaDeviceProp p;
+  cudaError_t e = cudaGetDeviceProperties(&p, device);
+  if (e != cudaSuccess) {
+    *why = std::string("cudaGetDeviceProperties: ") + cudaGetErrorString(e);
+    return e;
+  }
+  if (p.major != 10) {
+    *why = "device " + std::to_string(device) + " is sm_" + std::to_string(p.major) + std::to_string(p.minor) +
+           "; libjitc is built for sm_100a only";
+    return cudaErrorNoKernelImageForDevice;
+  }
+  cudaFuncAttributes fa;
+  e = cudaFuncGetAttributes(&fa, seg_kernel<kDigest>);
+  if (e != cudaSuccess) *why = std::string("sm_100a kernels not loadable: ") + cudaGetErrorString(e);
+  return e;
+}
+
+cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig, int grid,
+                            cudaStream_t s) {
+  uint32_t total = r.prefix[r.n];
+  if (total == 0) return cudaSuccess;
+  int g = (int)(total < (uint32_t)grid ? total : (uint32_t)grid);
+  auto* dig = reinterpret_cast<unsigned long long*>(d_dig);
+  switch (mode) {
+    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig); break;
+    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig); break;
+    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_phase_write(uint64_t* dev_slot, uint64_t value, cudaStream_t s) {
+  phase_write_kernel<<<1, 1, 0, s>>>(dev_slot, value);
+  return cudaGetLastError();
+}
+
+}  // namespace jitc
+
+using namespace jitc;
+
+static uint64_t host_mix(uint64_t x) { return jitc::mix64(x); }
+
+extern "C" {
+
+jitc_status jitc_gen_fill(void* dptr, uint32_t dtype, uint64_t numel, uint64_t seed, uint32_t group,
+                          uint32_t gen_id, uint32_t exp_lo, uint32_t exp_hi, int32_t force_pos, void* stream) {
+  if (!dptr && numel) { set_error("jitc_gen_fill: null pointer"); return JITC_EINVAL; }
+  if (dtype > 4 || exp_hi < exp_lo || exp_hi > 254) { set_error("jitc_gen_fill: bad dtype/range"); return JITC_EINVAL; }
+  if (!numel) return JITC_OK;
+  uint64_t key = host_mix(((uint64_t)group << 48) ^ ((uint64_t)gen_id << 32));
+  int grid = 148 * 8;
+  gen_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>((uint8_t*)dptr, dtype, numel, seed, key, exp_lo,
+                                                     exp_hi - exp_lo + 1, force_pos);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) { set_error(std::string("jitc_gen_fill: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
+  return JITC_OK;
+}
+
+jitc_status jitc_inject_update(void* dptr, uint64_t e0, uint64_t count, uint32_t gen_id, uint64_t v, void* stream) {
+  if (!dptr && count) { set_error("jitc_inject_update: null pointer"); return JITC_EINVAL; }
+  if (!count) return JITC_OK;
+  update_kernel<<<148 * 8, 256, 0, (cudaStream_t)stream>>>((uint32_t*)dptr, e0, count, (uint64_t)gen_id << 40,
+                                                            v * PHI);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) { set_error(std::string("jitc_inject_update: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
+  return JITC_OK;
+}
+
+jitc_status jitc_inject_rne(const void* master, void* param, uint64_t count, void* stream) {
+  if ((!master || !param) && count) { set_error("jitc_inject_rne: null pointer"); return JITC_EINVAL; }
+  if (!count) return JITC_OK;
+  rne_kernel<<<148 * 8, 256, 0, (cudaStream_t)stream>>>((const uint32_t*)master, (uint16_t*)param, count);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) { set_error(std::string("jitc_inject_rne: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
+  return JITC_OK;
+}
+
+jitc_status jitc_inject_bitflip(void* dptr, uint64_t byte, uint32_t bit, void* stream) {
+  if (!dptr || bit > 7) { set_error("jitc_inject_bitflip: bad argument"); return JITC_EINVAL; }
+  bitflip_kernel<<<1, 1, 0, (cudaStream_t)stream>>>((uint8_t*)dptr + byte, (uint8_t)(1u << bit));
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) { set_error(std::string("jitc_inject_bitflip: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
+  return JITC_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,323 @@
+"""Thin Python binding of libjitc.so (include/jitc.h): argument marshalling
+only -- every step of the path runs in the library's C++/CUDA code.
+
+The binding never falls back to anything: if libjitc.so is missing or the GPU
+is not an sm_100 part, the calls raise.  PyTorch is used by callers only for
+device memory, streams and process groups.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import struct
+from typing import Dict, List, Optional, Sequence, Tuple
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+SO_PATH = os.path.join(_PKG, "libjitc.so")
+
+OK, EINVAL, ESTATE, ENOMEM, ECUDA, ENCCL = 0, -1, -2, -3, -4, -5
+ELAYOUT, ENOREPLICA, ECONFLICT, ENOCONSISTENT = -6, -7, -8, -9
+EUNSTABLE, ECORRUPT, EINCOMPLETE, EIO = -10, -11, -12, -13
+STATUS_NAMES = {v: k for k, v in dict(
+    OK=OK, EINVAL=EINVAL, ESTATE=ESTATE, ENOMEM=ENOMEM, ECUDA=ECUDA, ENCCL=ENCCL, ELAYOUT=ELAYOUT,
+    ENOREPLICA=ENOREPLICA, ECONFLICT=ECONFLICT, ENOCONSISTENT=ENOCONSISTENT, EUNSTABLE=EUNSTABLE,
+    ECORRUPT=ECORRUPT, EINCOMPLETE=EINCOMPLETE, EIO=EIO).items()}
+CLEAN, DIRTY = 0, 1
+REQUIRED, OPTIONAL = 0, 1
+HOST, PEER = 0, 1
+ALL_GROUPS = 0xFFFFFFFF
+F_ZERO_COPY_D2H, F_ZERO_COPY_H2D, F_TIME_KERNELS, F_NO_SHM_UNLINK = 1, 2, 4, 8
+K_DIGEST, K_PACK, K_UNPACK = 1, 2, 3
+
+
+class JitcError(RuntimeError):
+    def __init__(self, status: int, msg: str, first_bad: int = -1):
+        super().__init__(f"{STATUS_NAMES.get(status, status)}: {msg}")
+        self.status = status
+        self.first_bad = first_bad
+
+
+class Config(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("flags", ctypes.c_uint32), ("chunk_bytes", ctypes.c_uint64), ("staging", ctypes.c_void_p),
+                ("staging_bytes", ctypes.c_uint64), ("slot_bytes", ctypes.c_uint64),
+                ("image_dir", ctypes.c_char_p), ("streams", ctypes.c_void_p * 2)]
+
+
+class Tensor(ctypes.Structure):
+    _fields_ = [("name", ctypes.c_char_p), ("ptr", ctypes.c_void_p), ("nbytes", ctypes.c_uint64),
+                ("dtype", ctypes.c_uint32)]
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [("ms_host", ctypes.c_double), ("ms_device", ctypes.c_double), ("ms_kernel", ctypes.c_double),
+                ("image_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64), ("h2d_bytes", ctypes.c_uint64),
+                ("p2p_bytes", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64), ("rounds", ctypes.c_uint32),
+                ("first_bad_chunk", ctypes.c_int32)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class KernelCounter(ctypes.Structure):
+    _fields_ = [("launches", ctypes.c_uint64), ("bytes", ctypes.c_uint64), ("ms", ctypes.c_double)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Loads the in-tree libjitc.so; raises if it has not been built."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(SO_PATH):
+        raise RuntimeError(f"{SO_PATH} not built: run `python -m paper_conf_eurosys_guptakkvgkrs24_b200.build` "
+                           "(there is no CPU fallback)")
+    L = ctypes.CDLL(SO_PATH)
+    i32, u32, u64, vp, sz = ctypes.c_int32, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_size_t
+    P = ctypes.POINTER
+    sig = {
+        "jitc_create": ([P(Config), P(vp)], i32),
+        "jitc_destroy": ([vp], None),
+        "jitc_last_error": ([vp], ctypes.c_char_p),
+        "jitc_abi_version": ([], ctypes.c_int),
+        "jitc_register": ([vp, u32, i32, P(i32), i32, P(Tensor), sz, P(u64), P(u64)], i32),
+        "jitc_declare_group": ([vp, u32, i32, P(i32), i32], i32),
+        "jitc_mark": ([vp, u32, u64, i32, vp], i32),
+        "jitc_phase": ([vp, u32, P(u64), P(i32)], i32),
+        "jitc_get_unique_id": ([vp], i32),
+        "jitc_comm_init": ([vp, vp, i32, i32, P(i32)], i32),
+        "jitc_comm_shrink": ([vp, P(i32), i32], i32),
+        "jitc_comm_destroy": ([vp], i32),
+        "jitc_fingerprint": ([vp, u32, vp, sz, P(sz)], i32),
+        "jitc_exchange_records": ([vp, vp, sz, vp, sz, P(sz)], i32),
+        "jitc_select_consistent_replica": ([vp, sz, P(i32), i32, vp, sz, P(sz)], i32),
+        "jitc_capture": ([vp, vp, sz, u32, P(Stats)], i32),
+        "jitc_commit": ([vp, vp, sz], i32),
+        "jitc_restore": ([vp, u32, i32, vp, sz, P(Stats)], i32),
+        "jitc_verify": ([vp, u32, vp, sz, P(u64)], i32),
+        "jitc_layout": ([P(Tensor), sz, u64, P(u64), P(u64), P(u64)], i32),
+        "jitc_shard_range": ([u64, u32, u32, P(u64), P(u64)], i32),
+        "jitc_kernel_counters": ([vp, i32, P(KernelCounter)], i32),
+        "jitc_reset_counters": ([vp], i32),
+        "jitc_gen_fill": ([vp, u32, u64, u64, u32, u32, u32, u32, i32, vp], i32),
+        "jitc_inject_update": ([vp, u64, u64, u32, u64, vp], i32),
+        "jitc_inject_rne": ([vp, vp, u64, vp], i32),
+        "jitc_inject_bitflip": ([vp, u64, u32, vp], i32),
+    }
+    for name, (args, res) in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = res
+    _lib = L
+    return L
+
+
+EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version", "jitc_register",
+            "jitc_declare_group", "jitc_mark", "jitc_phase", "jitc_get_unique_id", "jitc_comm_init",
+            "jitc_comm_shrink", "jitc_comm_destroy", "jitc_fingerprint", "jitc_exchange_records",
+            "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
+            "jitc_layout", "jitc_shard_range", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
+            "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip"]
+
+
+def last_error() -> str:
+    return lib().jitc_last_error(None).decode(errors="replace")
+
+
+def _check(st: int, what: str, first_bad: int = -1):
+    if st != OK:
+        raise JitcError(st, f"{what}: {last_error()}", first_bad)
+
+
+def _i32arr(xs: Sequence[int]):
+    return (ctypes.c_int32 * max(len(xs), 1))(*xs)
+
+
+# ------------------------------------------------------------------ pure calls
+def layout(tensors: Sequence[Tuple[str, int, int]], chunk_bytes: int) -> Tuple[List[int], int, int]:
+    """O1 through the C ABI: [(name, nbytes, dtype)] -> (offsets, layout_hash, L)."""
+    n = len(tensors)
+    names = [t[0].encode() for t in tensors]
+    arr = (Tensor * max(n, 1))(*[Tensor(nm, None, nb, dt) for nm, (_, nb, dt) in zip(names, tensors)])
+    offs = (ctypes.c_uint64 * max(n, 1))()
+    lh, L = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(lib().jitc_layout(arr, n, chunk_bytes, offs, ctypes.byref(lh), ctypes.byref(L)), "jitc_layout")
+    return list(offs)[:n], lh.value, L.value
+
+
+def shard_range(n_c: int, k: int, s: int) -> Tuple[int, int]:
+    a, b = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(lib().jitc_shard_range(n_c, k, s, ctypes.byref(a), ctypes.byref(b)), "jitc_shard_range")
+    return a.value, b.value
+
+
+def select_consistent_replica(blobs: bytes, healthy: Sequence[int]) -> Tuple[int, bytes]:
+    """Returns (status, selection bytes); the selection is written on every status."""
+    L = lib()
+    n = ctypes.c_size_t()
+    h = _i32arr(list(healthy))
+    L.jitc_select_consistent_replica(blobs, len(blobs), h, len(healthy), None, 0, ctypes.byref(n))
+    buf = ctypes.create_string_buffer(n.value)
+    st = L.jitc_select_consistent_replica(blobs, len(blobs), h, len(healthy), buf, n.value, ctypes.byref(n))
+    return st, buf.raw[:n.value]
+
+
+def parse_selection(sel: bytes) -> dict:
+    """Decodes a selection blob for inspection."""
+    magic, fmt, n_groups, status, bad_group, v_star, topo_hash, sel_bytes, _ = struct.unpack_from("<IHHiiQQQQ", sel, 0)
+    out = dict(status=status, bad_group=bad_group, v_star=v_star, topo_hash=topo_hash, groups=[])
+    q = 48
+    for _ in range(n_groups):
+        (group, policy, gst, k, n_mem, n_ex, n_cf, _r, lh, C, n_c, L, root) = struct.unpack_from("<IBBHIIIIQQQQQ", sel, q)
+        q += 64
+        ints = struct.unpack_from(f"<{k + n_mem + 2 * n_ex}i", sel, q)
+        q += 4 * len(ints)
+        q += (-q) % 8
+        cf = list(struct.unpack_from(f"<{n_cf}Q", sel, q))
+        q += 8 * n_cf
+        out["groups"].append(dict(group=group, policy=policy, status=gst, writers=list(ints[:k]),
+                                  members=list(ints[k:k + n_mem]),
+                                  excluded=[(ints[k + n_mem + 2 * j], ints[k + n_mem + 2 * j + 1]) for j in range(n_ex)],
+                                  conflict_chunks=cf, layout_hash=lh, chunk_bytes=C, n_c=n_c, image_bytes=L, root=root))
+    return out
+
+
+def get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().jitc_get_unique_id(buf), "jitc_get_unique_id")
+    return buf.raw
+
+
+# ------------------------------------------------------------------ K4 harness kernels
+def gen_fill(ptr: int, dtype: int, numel: int, seed: int, group: int, gen_id: int, lo: int, hi: int, pos: bool,
+             stream: int = 0):
+    _check(lib().jitc_gen_fill(ptr, dtype, numel, seed, group, gen_id, lo, hi, int(pos), stream or None),
+           "jitc_gen_fill")
+
+
+def inject_update(ptr: int, e0: int, count: int, gen_id: int, v: int, stream: int = 0):
+    _check(lib().jitc_inject_update(ptr, e0, count, gen_id, v, stream or None), "jitc_inject_update")
+
+
+def inject_rne(master_ptr: int, param_ptr: int, count: int, stream: int = 0):
+    _check(lib().jitc_inject_rne(master_ptr, param_ptr, count, stream or None), "jitc_inject_rne")
+
+
+def inject_bitflip(ptr: int, byte: int, bit: int, stream: int = 0):
+    _check(lib().jitc_inject_bitflip(ptr, byte, bit, stream or None), "jitc_inject_bitflip")
+
+
+# ------------------------------------------------------------------ context
+class Context:
+    """One libjitc context (one GPU, one process).  Methods map 1:1 to the C ABI."""
+
+    def __init__(self, device: int = 0, rank: int = 0, world: int = 1, chunk_bytes: int = 1 << 20,
+                 staging_bytes: int = 0, slot_bytes: int = 0, image_dir: Optional[str] = None, flags: int = 0,
+                 staging_ptr: int = 0, streams: Tuple[int, int] = (0, 0)):
+        self._L = lib()
+        self._image_dir = image_dir.encode() if image_dir else None
+        cfg = Config(device, rank, world, flags, chunk_bytes, staging_ptr or None, staging_bytes, slot_bytes,
+                     self._image_dir, (ctypes.c_void_p * 2)(streams[0] or None, streams[1] or None))
+        h = ctypes.c_void_p()
+        _check(self._L.jitc_create(ctypes.byref(cfg), ctypes.byref(h)), "jitc_create")
+        self._h = h
+        self.rank, self.world = rank, world
+        self._keep = []   # tensors registered (caller-owned, must stay alive)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._L.jitc_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -- steady state
+    def register(self, group: int, policy: int, members: Sequence[int], tensors: Sequence[Tuple[str, int, int, int]],
+                 keepalive=None) -> Tuple[int, int]:
+        """tensors: [(name, device_ptr, nbytes, dtype)] -> (layout_hash, image_bytes)."""
+        names = [t[0].encode() for t in tensors]
+        arr = (Tensor * max(len(tensors), 1))(*[Tensor(nm, p or None, nb, dt)
+                                                for nm, (_, p, nb, dt) in zip(names, tensors)])
+        lh, L = ctypes.c_uint64(), ctypes.c_uint64()
+        m = _i32arr(list(members))
+        _check(self._L.jitc_register(self._h, group, policy, m, len(members), arr, len(tensors), ctypes.byref(lh),
+                                     ctypes.byref(L)), "jitc_register")
+        if keepalive is not None:
+            self._keep.append(keepalive)
+        return lh.value, L.value
+
+    def declare_group(self, group: int, policy: int, members: Sequence[int]):
+        _check(self._L.jitc_declare_group(self._h, group, policy, _i32arr(list(members)), len(members)),
+               "jitc_declare_group")
+
+    def mark(self, group: int, version: int, phase: int, stream: int = 0):
+        _check(self._L.jitc_mark(self._h, group, version, phase, stream or None), "jitc_mark")
+
+    def phase(self, group: int) -> Tuple[int, int]:
+        v, p = ctypes.c_uint64(), ctypes.c_int32()
+        _check(self._L.jitc_phase(self._h, group, ctypes.byref(v), ctypes.byref(p)), "jitc_phase")
+        return v.value, p.value
+
+    # -- communicator
+    def comm_init(self, uid: bytes, nranks: int, comm_rank: int, job_ranks: Optional[Sequence[int]] = None):
+        jr = _i32arr(list(job_ranks)) if job_ranks is not None else None
+        _check(self._L.jitc_comm_init(self._h, uid, nranks, comm_rank, jr), "jitc_comm_init")
+
+    def comm_shrink(self, failed: Sequence[int]):
+        _check(self._L.jitc_comm_shrink(self._h, _i32arr(list(failed)), len(failed)), "jitc_comm_shrink")
+
+    def comm_destroy(self):
+        _check(self._L.jitc_comm_destroy(self._h), "jitc_comm_destroy")
+
+    # -- capture
+    def fingerprint(self, group: int = ALL_GROUPS) -> bytes:
+        n = ctypes.c_size_t()
+        _check(self._L.jitc_fingerprint(self._h, group, None, 0, ctypes.byref(n)), "jitc_fingerprint")
+        buf = ctypes.create_string_buffer(n.value)
+        _check(self._L.jitc_fingerprint(self._h, group, buf, n.value, ctypes.byref(n)), "jitc_fingerprint")
+        return buf.raw[:n.value]
+
+    def exchange_records(self, mine: bytes) -> bytes:
+        n = ctypes.c_size_t()
+        _check(self._L.jitc_exchange_records(self._h, mine, len(mine), None, 0, ctypes.byref(n)),
+               "jitc_exchange_records")
+        buf = ctypes.create_string_buffer(max(n.value, 1))
+        _check(self._L.jitc_exchange_records(self._h, mine, len(mine), buf, n.value, ctypes.byref(n)),
+               "jitc_exchange_records")
+        return buf.raw[:n.value]
+
+    def capture(self, selection: bytes, group: int = ALL_GROUPS) -> dict:
+        st = Stats()
+        _check(self._L.jitc_capture(self._h, selection, len(selection), group, ctypes.byref(st)), "jitc_capture")
+        return st.as_dict()
+
+    def commit(self, selection: bytes):
+        _check(self._L.jitc_commit(self._h, selection, len(selection)), "jitc_commit")
+
+    # -- restore
+    def restore(self, group: int = ALL_GROUPS, mode: int = HOST, selection: Optional[bytes] = None) -> dict:
+        st = Stats()
+        r = self._L.jitc_restore(self._h, group, mode, selection, len(selection) if selection else 0, ctypes.byref(st))
+        _check(r, "jitc_restore", st.first_bad_chunk)
+        return st.as_dict()
+
+    def verify(self, group: int, expected: Optional[bytes] = None) -> int:
+        """Returns UINT64_MAX on success; raises JitcError(ECORRUPT) with first_bad on mismatch."""
+        fb = ctypes.c_uint64()
+        r = self._L.jitc_verify(self._h, group, expected, len(expected) if expected else 0, ctypes.byref(fb))
+        _check(r, "jitc_verify", fb.value if r == ECORRUPT else -1)
+        return fb.value
+
+    def kernel_counters(self, kind: int) -> dict:
+        kc = KernelCounter()
+        _check(self._L.jitc_kernel_counters(self._h, kind, ctypes.byref(kc)), "jitc_kernel_counters")
+        return dict(launches=kc.launches, bytes=kc.bytes, ms=kc.ms)
+
+    def reset_counters(self):
+        _check(self._L.jitc_reset_counters(self._h), "jitc_reset_counters")

@@ -1,0 +1,306 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  All of this is integer / byte work, so the bar is
+bit-exact (BASELINE.json north_star)."""
+import os
+import shutil
+import uuid
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import oracle as O
+from workloads import configs as W
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def J():
+    from paper_conf_eurosys_guptakkvgkrs24_b200 import build, jitc
+    build.build()
+    assert torch.cuda.is_available(), "GPU tests need a B200"
+    return jitc
+
+
+@pytest.fixture
+def shm():
+    d = f"/dev/shm/jitc-test-{os.getpid()}-{uuid.uuid4().hex[:8]}"
+    yield d
+    shutil.rmtree(d, ignore_errors=True)
+
+
+def _state(g, seed, **kw):
+    from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
+    return GroupState(g, seed, **kw)
+
+
+def _ctx(J, C, image_dir=None, flags=0, staging=64 << 20, slot=8 << 20, rank=0, world=1):
+    return J.Context(device=0, rank=rank, world=world, chunk_bytes=C, staging_bytes=staging, slot_bytes=slot,
+                     image_dir=image_dir, flags=flags | J.F_TIME_KERNELS)
+
+
+def _records(blob):
+    [(rank, topo, th, recs)] = O.decode_blobs(blob)
+    return {r.group: r for r in recs}
+
+
+def _small_groups():
+    gs = [W.random_table(s, 60, max_bytes=20000, group=s) for s in range(3)]
+    gs.append(W.scaled(W.c2(), 40000).groups[0])
+    gs[-1].group = 7
+    return gs
+
+
+# ------------------------------------------------------------------ K4 generator
+def test_k4_generator_matches_oracle(J):
+    for g in _small_groups()[:2] + [W.c1().groups[0]]:
+        st = _state(g, 0x1234)
+        torch.cuda.synchronize()
+        for i, t in enumerate(g.tensors):
+            got = st.tensor_bytes(i).cpu().numpy()
+            want = O.gen_tensor_bytes(t, 0x1234, g.group)
+            assert np.array_equal(got, want), t.name
+
+
+def test_k4_update_and_rne_match_oracle(J):
+    g = W.c1().groups[0]
+    st = _state(g, 7)
+    L = O.lib()
+    for i in (0, 5, 60):
+        t = g.tensors[i]
+        x = st.tensor_bytes(i)
+        J.inject_update(x.data_ptr(), 3, t.numel - 3, t.gen_id, 11)
+        torch.cuda.synchronize()
+        want = O.gen_tensor_bytes(t, 7, g.group).view(np.uint32).copy()
+        L.orc_update_fp32(O._ptr(want[3:]), 3, t.numel - 3, t.gen_id, 11)
+        assert np.array_equal(x.cpu().numpy().view(np.uint32), want)
+        p = torch.empty(t.numel, dtype=torch.int16, device="cuda")
+        J.inject_rne(x.data_ptr(), p.data_ptr(), t.numel)
+        torch.cuda.synchronize()
+        ref = torch.from_numpy(want.view(np.float32).copy()).to(torch.bfloat16).view(torch.int16)
+        assert torch.equal(p.cpu(), ref)
+
+
+# ------------------------------------------------------------------ K1 fingerprint
+@pytest.mark.parametrize("C", [4096, 1 << 20])
+@pytest.mark.parametrize("misalign", [0, 2, 8])
+def test_k1_digests_match_oracle(J, C, misalign):
+    for g in _small_groups():
+        st = _state(g, 99, misalign=misalign)
+        ctx = _ctx(J, C)
+        lh, L = ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+        lay = O.layout_of_group(g, C)
+        assert (lh, L) == (lay.layout_hash, lay.L)
+        ctx.mark(g.group, 5, J.CLEAN)
+        rec = _records(ctx.fingerprint(g.group))[g.group]
+        img = O.pack(O.gen_group(g, 99), lay)
+        d = O.jf64(img, C, 0, lay.n_c)
+        assert np.array_equal(rec.d, d)
+        assert rec.root == O.root(lay.layout_hash, d) and rec.version == 5 and rec.phase == O.CLEAN
+        ctx.close()
+
+
+def test_k1_c1_full(J):
+    w = W.c1()
+    g = w.groups[0]
+    st = _state(g, w.seed)
+    ctx = _ctx(J, 1 << 20)
+    ctx.register(0, J.REQUIRED, [0, 1], st.table(), keepalive=st)
+    rec = _records(ctx.fingerprint())[0]
+    lay = O.layout_of_group(g, 1 << 20)
+    d = O.jf64(O.pack(O.gen_group(g, w.seed), lay), lay.C, 0, lay.n_c)
+    assert lay.L == 48_138_240 and np.array_equal(rec.d, d)
+
+
+def test_phase_word_stream_ordered(J):
+    g = W.random_table(1, 4)
+    st = _state(g, 1)
+    ctx = _ctx(J, 4096)
+    ctx.register(0, J.REQUIRED, [0], st.table(), keepalive=st)
+    s = torch.cuda.Stream()
+    ctx.mark(0, 41, J.DIRTY, s.cuda_stream)
+    s.synchronize()
+    assert ctx.phase(0) == (41, J.DIRTY)
+    ctx.mark(0, 42, J.CLEAN, s.cuda_stream)
+    s.synchronize()
+    assert ctx.phase(0) == (42, J.CLEAN)
+    ctx.mark(0, 43, J.DIRTY)          # host write
+    assert ctx.phase(0) == (43, J.DIRTY)
+    rec = _records(ctx.fingerprint())[0]
+    assert (rec.version, rec.phase) == (43, O.DIRTY)
+
+
+# ------------------------------------------------------------------ capture / restore
+def _pipeline(J, ctx, healthy=(0,)):
+    blob = ctx.fingerprint()
+    allb = ctx.exchange_records(blob)
+    st, sel = J.select_consistent_replica(allb, list(healthy))
+    assert st == J.OK, J.parse_selection(sel)
+    cap = ctx.capture(sel)
+    ctx.commit(sel)
+    return blob, sel, cap
+
+
+@pytest.mark.parametrize("flags", [0, 1, 2, 3])     # staging+CE / zero-copy D2H / zero-copy H2D / both
+@pytest.mark.parametrize("C", [4096, 1 << 20])
+def test_capture_restore_bit_exact(J, shm, flags, C):
+    for g in _small_groups():
+        st = _state(g, 5, misalign=2 if g.group == 1 else 0)
+        ctx = _ctx(J, C, image_dir=shm, flags=flags, staging=4 * C * 4, slot=4 * C)
+        ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+        ctx.mark(g.group, 3, J.CLEAN)
+        blob, sel, cap = _pipeline(J, ctx)
+        lay = O.layout_of_group(g, C)
+        want = O.pack(O.gen_group(g, 5), lay)
+        img = np.fromfile(f"{shm}/g{g.group}.img", dtype=np.uint8)[:lay.L]
+        assert np.array_equal(img, want)                       # K2 image == oracle pack
+        assert cap["image_bytes"] == lay.L and cap["kernel_launches"] >= 1
+        st.scramble()
+        res = ctx.restore(g.group, J.HOST)
+        torch.cuda.synchronize()
+        for i, t in enumerate(g.tensors):                      # K3 restore == original state
+            assert np.array_equal(st.tensor_bytes(i).cpu().numpy(), O.gen_tensor_bytes(t, 5, g.group)), t.name
+        assert ctx.verify(g.group) == 2**64 - 1
+        assert ctx.verify(g.group, blob) == 2**64 - 1
+        ctx.close()
+
+
+def test_restore_in_fresh_context_from_shm(J, shm):
+    """A replacement process registers the same tensors and restores from the
+    committed shared image (HOST mode, selection from the manifest)."""
+    g = W.scaled(W.c1(), 5000).groups[0]
+    st = _state(g, 8)
+    ctx = _ctx(J, 4096, image_dir=shm)
+    ctx.register(0, J.REQUIRED, [0, 1], st.table(), keepalive=st)
+    ctx.mark(0, 9, J.CLEAN)
+    _pipeline(J, ctx)
+    ctx.close()
+    st2 = _state(g, 8, fill=False, shuffle_seed=9)
+    st2.scramble()
+    ctx2 = _ctx(J, 4096, image_dir=shm, rank=1, world=2)
+    ctx2.register(0, J.REQUIRED, [0, 1], st2.table(), keepalive=st2)
+    ctx2.restore(0, J.HOST)
+    torch.cuda.synchronize()
+    for i, t in enumerate(g.tensors):
+        assert np.array_equal(st2.tensor_bytes(i).cpu().numpy(), O.gen_tensor_bytes(t, 8, 0))
+
+
+def test_corrupt_host_image_exact_chunk(J, shm):
+    g = _small_groups()[3]
+    C = 4096
+    st = _state(g, 6)
+    ctx = _ctx(J, C, image_dir=shm)
+    ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+    _pipeline(J, ctx)
+    lay = O.layout_of_group(g, C)
+    rng = np.random.default_rng(1)
+    for _ in range(5):
+        pos = int(rng.integers(0, lay.L))
+        with open(f"{shm}/g{g.group}.img", "r+b") as f:
+            f.seek(pos); b = f.read(1); f.seek(pos); f.write(bytes([b[0] ^ 0x10]))
+        with pytest.raises(J.JitcError) as e:
+            ctx.restore(g.group, J.HOST)
+        assert e.value.status == J.ECORRUPT and e.value.first_bad == pos // C
+        with open(f"{shm}/g{g.group}.img", "r+b") as f:
+            f.seek(pos); f.write(b)
+    ctx.restore(g.group, J.HOST)
+
+
+def test_uncommitted_refused(J, shm):
+    g = W.random_table(4, 10)
+    st = _state(g, 6)
+    ctx = _ctx(J, 4096, image_dir=shm)
+    ctx.register(0, J.REQUIRED, [0], st.table(), keepalive=st)
+    _pipeline(J, ctx)
+    os.unlink(f"{shm}/g0.commit")
+    with pytest.raises(J.JitcError) as e:
+        ctx.restore(0, J.HOST)
+    assert e.value.status == J.EINCOMPLETE
+
+
+def test_hbm_bitflip_detected_by_verify(J):
+    g = _small_groups()[3]
+    C = 4096
+    st = _state(g, 2)
+    ctx = _ctx(J, C)
+    ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+    blob = ctx.fingerprint()
+    lay = O.layout_of_group(g, C)
+    for i in (0, 3, len(g.tensors) - 1):
+        nb = g.tensors[i].nbytes
+        byte = nb // 2
+        J.inject_bitflip(st.ptrs[i], byte, 5)
+        with pytest.raises(J.JitcError) as e:
+            ctx.verify(g.group, blob)
+        assert e.value.status == J.ECORRUPT and e.value.first_bad == (lay.offsets[i] + byte) // C
+        J.inject_bitflip(st.ptrs[i], byte, 5)
+    ctx.verify(g.group, blob)
+
+
+def test_unstable_between_fingerprint_and_capture(J, shm):
+    g = _small_groups()[0]
+    st = _state(g, 2)
+    ctx = _ctx(J, 4096, image_dir=shm)
+    ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+    blob = ctx.fingerprint()
+    st_, sel = J.select_consistent_replica(blob, [0])
+    J.inject_bitflip(st.ptrs[2], 0, 0)
+    with pytest.raises(J.JitcError) as e:
+        ctx.capture(sel)
+    assert e.value.status == J.EUNSTABLE
+
+
+def test_half_step_detected(J):
+    """A half-applied optimizer step (U_v on tensors [0, split)) changes exactly
+    the chunks the oracle predicts, and the replica class splits."""
+    g = W.scaled(W.c1(), 20000).groups[0]
+    C = 4096
+    a, b = _state(g, 3), _state(g, 3)
+    ctxa, ctxb = _ctx(J, C, rank=0, world=2), _ctx(J, C, rank=1, world=2)
+    ctxa.register(0, J.REQUIRED, [0, 1], a.table(), keepalive=a)
+    ctxb.register(0, J.REQUIRED, [0, 1], b.table(), keepalive=b)
+    split = 40
+    for i in range(split):
+        t = g.tensors[i]
+        J.inject_update(b.ptrs[i], 0, t.numel, t.gen_id, 4)
+    torch.cuda.synchronize()
+    ra, rb = _records(ctxa.fingerprint())[0], _records(ctxb.fingerprint())[0]
+    lay = O.layout_of_group(g, C)
+    touched = set()
+    for i in range(split):
+        touched |= set(range(lay.offsets[i] // C, (lay.offsets[i] + lay.nbytes[i] - 1) // C + 1))
+    assert set(np.nonzero(ra.d != rb.d)[0].tolist()) == touched
+    st, sel = J.select_consistent_replica(ctxa.fingerprint() + ctxb.fingerprint(), [0, 1])
+    assert st == J.ECONFLICT
+
+
+# ------------------------------------------------------------------ full size (sampled)
+@pytest.mark.slow
+def test_c2_full_size_sampled(J, shm):
+    """C2 (GPT-2 1.5B, 24.9 GB) in the launch configuration bench.py times:
+    K1 digests of sampled chunks equal the oracle's (computed chunk by chunk),
+    capture+restore round-trips, verify passes, sampled image bytes equal."""
+    w = W.c2()
+    C = 1 << 20
+    states = {g.group: _state(g, w.seed) for g in w.groups}
+    ctx = J.Context(device=0, chunk_bytes=C, image_dir=shm, flags=J.F_TIME_KERNELS)
+    for g in w.groups:
+        ctx.register(g.group, g.policy, [0], states[g.group].table(), keepalive=states[g.group])
+        ctx.mark(g.group, 100, J.CLEAN)
+    blob, sel, cap = _pipeline(J, ctx)
+    recs = _records(blob)
+    rng = np.random.default_rng(0)
+    for g in w.groups:
+        lay = O.layout_of_group(g, C)
+        chunks = sorted(set([0, lay.n_c - 1] + rng.integers(0, lay.n_c, 12).tolist()))
+        img = np.memmap(f"{shm}/g{g.group}.img", dtype=np.uint8, mode="r")
+        for c in chunks:
+            a, b = c * C, min((c + 1) * C, lay.L)
+            want = O.image_range(g, w.seed, lay, a, b)
+            assert np.array_equal(np.asarray(img[a:b]), want)
+            assert int(recs[g.group].d[c]) == int(O.jf64(want, C, a, lay.n_c)[c])
+        states[g.group].scramble()
+    ctx.restore(J.ALL_GROUPS, J.HOST)
+    for g in w.groups:
+        ctx.verify(g.group, blob)
