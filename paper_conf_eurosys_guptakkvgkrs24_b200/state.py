@@ -24,7 +24,12 @@ class GroupState:
         offs = [0] * len(sizes)
         pos = 0
         for i in order:
-            offs[i] = pos + (misalign if (misalign and i % 3 == 1) else 0)
+            # misaligned placement (tests): shift every third tensor by `misalign`
+            # bytes, rounded up to its element size (an fp32 tensor is never
+            # less than 4-byte aligned in a real program)
+            eb = ELEM_BYTES[g.tensors[i].dtype]
+            shift = 0 if not (misalign and i % 3 == 1) else (misalign if misalign % eb == 0 else eb)
+            offs[i] = pos + shift
             pos = (offs[i] + sizes[i] + align - 1) // align * align
         self.arena = torch.empty(max(pos, 1), dtype=torch.uint8, device=f"cuda:{device}")
         base = self.arena.data_ptr()

@@ -84,7 +84,7 @@ def test_k4_update_and_rne_match_oracle(J):
 
 # ------------------------------------------------------------------ K1 fingerprint
 @pytest.mark.parametrize("C", [4096, 1 << 20])
-@pytest.mark.parametrize("misalign", [0, 2, 8])
+@pytest.mark.parametrize("misalign", [0, 1, 2, 8])
 def test_k1_digests_match_oracle(J, C, misalign):
     for g in _small_groups():
         st = _state(g, 99, misalign=misalign)
