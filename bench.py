@@ -331,8 +331,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3"])
     ap.add_argument("--impl", default="jitc", choices=["jitc", "reference"])
-    ap.add_argument("--staging", type=int, default=1024, help="MiB of device staging")
-    ap.add_argument("--slot", type=int, default=256, help="MiB per pipeline round")
+    ap.add_argument("--staging", type=int, default=8192, help="MiB of device staging")
+    ap.add_argument("--slot", type=int, default=2048, help="MiB per pipeline round")
     ap.add_argument("--zero-copy", action="store_true")
     ap.add_argument("--image-dir", default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -15,7 +15,7 @@ namespace jitc {
 
 constexpr uint64_t kGolden = 0x9E3779B97F4A7C15ull;  // JF64 key step (2^64 / golden ratio)
 constexpr uint64_t kAlign = 256;                       // image alignment (reading R4)
-constexpr uint32_t kMaxSegBytes = 128u << 10;          // K1/K2/K3 work unit (data bytes)
+constexpr uint32_t kMaxSegBytes = 32u << 10;           // K1/K2/K3 work unit (data bytes)
 constexpr int kMaxPhaseSlots = 512;
 constexpr int kEventPool = 8192;
 

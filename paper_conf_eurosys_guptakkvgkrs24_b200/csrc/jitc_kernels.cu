@@ -13,11 +13,11 @@
 // wrap-around sum of its terms.  The sum is order-free, so every CTA adds its
 // partial into d[chunk] with a 64-bit atomic and the result is deterministic.
 //
-// Work unit: one Seg = one piece (<= 128 KiB) of one tensor that never crosses
-// a chunk boundary.  A persistent grid of CTAs strides over segments; inside
-// a segment every thread streams 16-byte vectors (4 loads in flight before
+// Work unit: one Seg = one piece (<= 32 KiB) of one tensor that never crosses
+// a chunk boundary.  Each CTA of a persistent grid takes an equal contiguous
+// run of segments; inside a segment every thread streams 16-byte vectors (4 loads in flight before
 // any use), hashes both words, optionally stores, and the warp reduces its
-// partial with shuffles before one atomicAdd per warp per segment.  Pure HBM
+// partial with shuffles before one atomicAdd per warp per chunk it touched.  Pure HBM
 // (or PCIe) streaming: no tensor cores, no shared-memory reuse (every byte is
 // touched once), so the design targets coalescing, MLP and a grid sized to
 // the SM count.
@@ -89,23 +89,53 @@ __device__ __forceinline__ uint64_t warp_sum(uint64_t v) {
   return v;
 }
 
+// Segment v of the launch's virtual concatenation of ranges.
+__device__ __forceinline__ const Seg* seg_at(const Seg* segs, const LaunchRanges& R, uint32_t v, int* r) {
+  int k = 0;
+  while (v >= R.prefix[k + 1]) ++k;
+  *r = k;
+  return segs + R.seg_begin[k] + (v - R.prefix[k]);
+}
+
+// Warp-reduce the partial digest and add it to the chunk's digest.
+__device__ __forceinline__ void flush(unsigned long long* dig, uint32_t chunk, uint64_t acc, int lane) {
+  acc = warp_sum(acc);
+  if (lane == 0) atomicAdd(dig + chunk, (unsigned long long)acc);
+}
+
+// Every CTA takes a contiguous, equal-count run of segments (segments are
+// <= 32 KiB, so runs are balanced to within one segment), prefetches the
+// next descriptor while streaming the current one, and keeps the partial
+// digest in registers until the chunk changes.
 template <int MODE>
 __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ segs, LaunchRanges R,
                                                        unsigned long long* __restrict__ dig) {
   const uint32_t total = R.prefix[R.n];
+  const uint32_t v0 = (uint32_t)((uint64_t)blockIdx.x * total / gridDim.x);
+  const uint32_t v1 = (uint32_t)((uint64_t)(blockIdx.x + 1) * total / gridDim.x);
+  if (v0 >= v1) return;
   const int tid = threadIdx.x;
   const int lane = tid & 31;
-  for (uint32_t v = blockIdx.x; v < total; v += gridDim.x) {
-    int r = 0;
-    while (v >= R.prefix[r + 1]) ++r;
-    const Seg sg = segs[R.seg_begin[r] + (v - R.prefix[r])];
+  uint64_t acc = 0;
+  int r;
+  Seg next = *seg_at(segs, R, v0, &r);
+  int next_r = r;
+  uint32_t cur_chunk = next.chunk;
+  for (uint32_t v = v0; v < v1; ++v) {
+    const Seg sg = next;
+    r = next_r;
+    if (v + 1 < v1) next = *seg_at(segs, R, v + 1, &next_r);
+    if (sg.chunk != cur_chunk) {
+      flush(dig, cur_chunk, acc, lane);
+      acc = 0;
+      cur_chunk = sg.chunk;
+    }
     const uint64_t rel = sg.img_off - R.base_off[r];
     uint8_t* img = reinterpret_cast<uint8_t*>(R.base[r]) + rel;  // 16-B aligned (staging / host image)
     uint8_t* ten = reinterpret_cast<uint8_t*>(sg.src);
     const uint64_t data = sg.data_bytes;
     const uint64_t words = (data + sg.pad_bytes) >> 3;
     const uint64_t g0 = sg.img_off >> 3;
-    uint64_t acc = 0;
     uint64_t body_words = 0;
 
     if (sg.flags & kSegAligned16) {
@@ -156,9 +186,8 @@ __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ s
       }
       acc += dmix(x ^ ((g0 + w + 1ull) * PHI));
     }
-    acc = warp_sum(acc);
-    if (lane == 0) atomicAdd(dig + sg.chunk, (unsigned long long)acc);
   }
+  flush(dig, cur_chunk, acc, lane);
 }
 
 __global__ void phase_write_kernel(volatile uint64_t* slot, uint64_t value) {

@@ -31,7 +31,8 @@ def main(budget=int(os.environ.get("PROF_BYTES", 2 << 30)), reps=int(os.environ.
     g.tensors = keep
     shm = f"/dev/shm/jitc-prof-{os.getpid()}"
     st = GroupState(g, w.seed)
-    ctx = J.Context(device=0, chunk_bytes=1 << 20, staging_bytes=1 << 30, slot_bytes=256 << 20, image_dir=shm,
+    ctx = J.Context(device=0, chunk_bytes=1 << 20, staging_bytes=int(os.environ.get("PROF_STAGING_MB", 1024)) << 20,
+                    slot_bytes=int(os.environ.get("PROF_SLOT_MB", 256)) << 20, image_dir=shm,
                     flags=J.F_TIME_KERNELS | int(os.environ.get("PROF_FLAGS", "0")))
     ctx.register(0, J.REQUIRED, [0], st.table(), keepalive=st)
     ctx.mark(0, 1, J.CLEAN)
@@ -46,7 +47,9 @@ def main(budget=int(os.environ.get("PROF_BYTES", 2 << 30)), reps=int(os.environ.
     for k, n in ((1, "K1"), (2, "K2"), (3, "K3")):
         c = ctx.kernel_counters(k)
         rw = 1 if k == 1 else 2
-        print(n, c, "GB/s=%.1f" % (rw * c["bytes"] / (c["ms"] * 1e-3) / 1e9 if c["ms"] else 0))
+        print(n, "launches", c["launches"], "us/launch %.1f" % (1e3 * c["ms"] / max(c["launches"], 1)),
+              "MB/launch %.1f" % (c["bytes"] / max(c["launches"], 1) / 1e6),
+              "GB/s=%.1f" % (rw * c["bytes"] / (c["ms"] * 1e-3) / 1e9 if c["ms"] else 0))
     ctx.close()
     shutil.rmtree(shm, ignore_errors=True)
 
