@@ -36,7 +36,7 @@
  *    jitc_comm_init, jitc_comm_shrink, jitc_exchange_records, jitc_commit,
  *    jitc_restore.  Local: register, declare_group, mark, fingerprint,
  *    capture, verify.  Pure (no ctx, no GPU): jitc_layout, jitc_shard_range,
- *    jitc_select_consistent_replica.
+ *    jitc_select_consistent_replica, jitc_restore_plan.
  *  - No CPU fallback: if the device or the sm_100a kernels are unavailable
  *    the call fails with JITC_ECUDA.
  *  - Binary formats (record blob, selection, manifest, commit record) are
@@ -253,6 +253,18 @@ jitc_status jitc_layout(const jitc_tensor* t, size_t n, uint64_t chunk_bytes, ui
                         uint64_t* layout_hash, uint64_t* image_bytes);
 /* O5 shard rule: writer s of k gets chunks [*c0, *c1). */
 jitc_status jitc_shard_range(uint64_t n_c, uint32_t k, uint32_t s, uint64_t* c0, uint64_t* c1);
+/* The round schedule jitc_restore executes for `group` on comm rank
+ * `comm_rank` of an n-rank communicator whose comm rank i is job rank
+ * comm_job_ranks[i], given the staging geometry.  Output: a 24-B header
+ * ('JITP', n_ops, round_bytes, slots) followed by n_ops 48-B operations
+ * {round, kind (1 H2D, 2 ALLGATHER, 3 PACK, 4 SEND, 5 RECV, 6 UNPACK,
+ * 7 BCAST_DIGESTS), slot, peer, image range [a, b), staging offset, bytes}
+ * (DESIGN.md §8).  Pure: lets the multi-rank schedule be checked without
+ * GPUs.  cap == 0 => only *len. */
+jitc_status jitc_restore_plan(const void* selection, size_t sel_len, uint32_t group, int32_t mode,
+                              const int32_t* comm_job_ranks, int32_t n, int32_t comm_rank,
+                              uint64_t staging_bytes, uint64_t slot_bytes, void* plan, size_t cap,
+                              size_t* len);
 
 /* ---- counters ---------------------------------------------------------------- */
 jitc_status jitc_kernel_counters(jitc_ctx* ctx, int32_t kind, jitc_kernel_counter* out);

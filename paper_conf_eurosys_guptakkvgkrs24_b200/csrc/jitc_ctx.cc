@@ -947,6 +947,104 @@ static jitc_status compare_digests(jitc_ctx* c, GroupState& g, const std::vector
   return JITC_OK;
 }
 
+// Executes a restore plan (jitc_plan.cc) round by round: H2D on the copy
+// stream; K2 packs, NCCL send/recv or all-gather and K3 unpacks on the
+// compute stream; slot reuse ordered by the ready/free events.
+static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<PlanOp>& ops, uint32_t S,
+                                jitc_stats* stats) {
+  if (S > (uint32_t)jitc_ctx::kSlots) return fail(JITC_EINVAL, "execute_plan: too many slots");
+  bool used[jitc_ctx::kSlots] = {false};
+  size_t i = 0;
+  uint32_t rounds = 0;
+  while (i < ops.size()) {
+    if (ops[i].kind == kOpBcastDigests) {
+      ++i;
+      continue;
+    }
+    const uint32_t j = ops[i].round;
+    size_t e = i;
+    while (e < ops.size() && ops[e].round == j && ops[e].kind != kOpBcastDigests) ++e;
+    const uint32_t sl = ops[i].slot;
+    ++rounds;
+    // 1. host -> device on the copy stream
+    bool any_h2d = false;
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpH2D) continue;
+      if (!any_h2d && used[sl]) CU(cudaStreamWaitEvent(c->s_copy, c->ev_free[sl], 0));
+      any_h2d = true;
+      CU(cudaMemcpyAsync(c->staging + op.off, g.img_h + op.a, op.bytes, cudaMemcpyHostToDevice, c->s_copy));
+      if (stats) stats->h2d_bytes += op.bytes;
+    }
+    if (any_h2d) {
+      CU(cudaEventRecord(c->ev_ready[sl], c->s_copy));
+      CU(cudaStreamWaitEvent(c->s_comp, c->ev_ready[sl], 0));
+    }
+    // 2. K2 packs (PEER writers)
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpPack) continue;
+      uint32_t lo, hi;
+      seg_span(g, op.a, op.b, &lo, &hi);
+      jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, c->staging + op.off, op.a), g.d_dig2, op.b - op.a);
+      if (st) return st;
+    }
+    // 3. NCCL: point-to-point (PEER) and all-gather (HOST, n > 1)
+    bool p2p = false;
+    for (size_t q = i; q < e; ++q) p2p |= ops[q].kind == kOpSend || ops[q].kind == kOpRecv;
+    if (p2p) {
+      NC(ncclGroupStart());
+      for (size_t q = i; q < e; ++q) {
+        const PlanOp& op = ops[q];
+        if (op.kind == kOpSend) NC(ncclSend(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+        if (op.kind == kOpRecv) NC(ncclRecv(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+        if (stats) stats->p2p_bytes += op.bytes;
+      }
+      NC(ncclGroupEnd());
+    }
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpAllGather) continue;
+      uint8_t* base = c->staging + op.off;
+      NC(ncclAllGather(base + (uint64_t)c->comm_rank * op.bytes, base, op.bytes, ncclUint8, c->comm, c->s_comp));
+      if (stats) stats->p2p_bytes += (uint64_t)(c->comm_n - 1) * op.bytes;
+    }
+    // 4. K3 unpack + verify of every block of the round (<= kMaxRanges per launch)
+    LaunchRanges lr{};
+    uint64_t bytes = 0;
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpUnpack) continue;
+      uint32_t lo, hi;
+      seg_span(g, op.a, op.b, &lo, &hi);
+      add_range(lr, lo, hi, c->staging + op.off, op.a);
+      bytes += op.b - op.a;
+      if (lr.n == kMaxRanges) {
+        jitc_status st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
+        if (st) return st;
+        lr = LaunchRanges{};
+        bytes = 0;
+      }
+    }
+    if (lr.n) {
+      jitc_status st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
+      if (st) return st;
+    }
+    CU(cudaEventRecord(c->ev_free[sl], c->s_comp));
+    used[sl] = true;
+    i = e;
+  }
+  if (stats) stats->rounds += rounds;
+  return JITC_OK;
+}
+
+static jitc_status make_plan(jitc_ctx* c, const PlanInput& in, std::vector<PlanOp>* ops, uint32_t* S) {
+  uint64_t R;
+  std::string why;
+  if (!build_restore_plan(in, ops, &R, S, &why)) return fail(JITC_ENOMEM, "jitc_restore: " + why);
+  return JITC_OK;
+}
+
 // HOST mode: this rank (or, with a communicator, every comm rank) loads a
 // 1/n slice of the committed image H2D; slices are all-gathered over NVLink
 // round by round and every round is unpacked+verified by K3.
@@ -956,83 +1054,28 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
   if (st) return st;
   if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
   const int n = c->comm ? c->comm_n : 1;
-  const int me = c->comm ? c->comm_rank : 0;
   if (n > 1 && !g.img_shm)
     return fail(JITC_EINVAL, "jitc_restore: HOST mode across ranks needs a shared image_dir (use PEER mode)");
   if (n == 1 && (c->cfg.flags & JITC_F_ZERO_COPY_H2D)) {
     st = run_segments(c, g, kUnpack, one_range(0, (uint32_t)g.segs.size(), g.img_d, 0), g.d_dig2, g.L);
     if (st) return st;
     if (stats) stats->rounds += 1, stats->h2d_bytes += g.L;
-  } else if (n == 1) {
-    const uint64_t R = c->slot_bytes;
-    const int nslots = (int)std::min<uint64_t>(jitc_ctx::kSlots, c->staging_bytes / R);
-    uint32_t j = 0;
-    for (uint64_t a = 0; a < g.L; a += R, ++j) {
-      uint64_t b = std::min(a + R, g.L);
-      int sl = (int)(j % nslots);
-      uint8_t* slot = c->staging + sl * R;
-      if (j >= (uint32_t)nslots) CU(cudaStreamWaitEvent(c->s_copy, c->ev_free[sl], 0));
-      CU(cudaMemcpyAsync(slot, g.img_h + a, b - a, cudaMemcpyHostToDevice, c->s_copy));
-      CU(cudaEventRecord(c->ev_ready[sl], c->s_copy));
-      CU(cudaStreamWaitEvent(c->s_comp, c->ev_ready[sl], 0));
-      uint32_t lo, hi;
-      seg_span(g, a, b, &lo, &hi);
-      st = run_segments(c, g, kUnpack, one_range(lo, hi, slot, a), g.d_dig2, b - a);
-      if (st) return st;
-      CU(cudaEventRecord(c->ev_free[sl], c->s_comp));
-    }
-    if (stats) stats->rounds += j, stats->h2d_bytes += g.L;
   } else {
-    // per-rank slices O5(n_c, n, r); R bytes per rank per round
-    uint64_t R = c->staging_bytes / (2ull * n) / g.C * g.C;
-    if (R == 0) return fail(JITC_ENOMEM, "jitc_restore: staging too small for the all-gather rounds");
-    R = std::min<uint64_t>(R, c->slot_bytes);
-    std::vector<uint64_t> q0(n), q1(n);
-    uint64_t maxlen = 0;
-    for (int r = 0; r < n; ++r) {
-      uint64_t c0, c1;
-      shard_range(g.n_c, n, r, &c0, &c1);
-      q0[r] = std::min(c0 * g.C, g.L);
-      q1[r] = std::min(c1 * g.C, g.L);
-      maxlen = std::max(maxlen, q1[r] - q0[r]);
-    }
-    uint32_t J = (uint32_t)((maxlen + R - 1) / R);
-    for (uint32_t j = 0; j < J; ++j) {
-      int sl = (int)(j % 2);
-      uint8_t* buf = c->staging + (uint64_t)sl * n * R;
-      if (j >= 2) CU(cudaStreamWaitEvent(c->s_copy, c->ev_free[sl], 0));
-      uint64_t a = q0[me] + j * R, b = std::min(q1[me], a + R);
-      if (b > a) {
-        CU(cudaMemcpyAsync(buf + me * R, g.img_h + a, b - a, cudaMemcpyHostToDevice, c->s_copy));
-        if (stats) stats->h2d_bytes += b - a;
-      }
-      CU(cudaEventRecord(c->ev_ready[sl], c->s_copy));
-      CU(cudaStreamWaitEvent(c->s_comp, c->ev_ready[sl], 0));
-      NC(ncclAllGather(buf + me * R, buf, R, ncclUint8, c->comm, c->s_comp));
-      if (stats) stats->p2p_bytes += (uint64_t)(n - 1) * R;
-      LaunchRanges lr{};
-      uint64_t bytes = 0;
-      for (int r = 0; r < n; ++r) {
-        uint64_t ra = q0[r] + j * R, rb = std::min(q1[r], ra + R);
-        if (rb <= ra) continue;
-        uint32_t lo, hi;
-        seg_span(g, ra, rb, &lo, &hi);
-        add_range(lr, lo, hi, buf + r * R, ra);
-        bytes += rb - ra;
-        if (lr.n == kMaxRanges) {
-          st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
-          if (st) return st;
-          lr = LaunchRanges{};
-          bytes = 0;
-        }
-      }
-      if (lr.n) {
-        st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
-        if (st) return st;
-      }
-      CU(cudaEventRecord(c->ev_free[sl], c->s_comp));
-    }
-    if (stats) stats->rounds += J;
+    PlanInput in;
+    in.mode = JITC_RESTORE_HOST;
+    in.n_c = g.n_c;
+    in.chunk_bytes = g.C;
+    in.image_bytes = g.L;
+    in.n = n;
+    in.me = c->comm ? c->comm_rank : 0;
+    in.staging_bytes = c->staging_bytes;
+    in.slot_bytes = c->slot_bytes;
+    std::vector<PlanOp> ops;
+    uint32_t S = 0;
+    st = make_plan(c, in, &ops, &S);
+    if (st) return st;
+    st = execute_plan(c, g, ops, S, stats);
+    if (st) return st;
   }
   st = compare_digests(c, g, mv.d, stats);
   if (st) return st;
@@ -1051,114 +1094,62 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   if (gs.writers.empty()) return JITC_OK;  // dropped OPTIONAL group
   if (gs.layout_hash != g.layout_hash || gs.n_c != g.n_c || gs.image_bytes != g.L)
     return fail(JITC_ELAYOUT, "jitc_restore: selection layout differs from the registered one");
-  const int k = (int)gs.writers.size();
-  std::vector<int> wc(k);
-  for (int s = 0; s < k; ++s) {
-    wc[s] = comm_rank_of(c, gs.writers[s]);
-    if (wc[s] < 0) return fail(JITC_EINVAL, "jitc_restore: a writer is not in the communicator");
+  PlanInput in;
+  in.mode = JITC_RESTORE_PEER;
+  in.n_c = g.n_c;
+  in.chunk_bytes = g.C;
+  in.image_bytes = g.L;
+  in.n = c->comm_n;
+  in.me = c->comm_rank;
+  in.staging_bytes = c->staging_bytes;
+  in.slot_bytes = c->slot_bytes;
+  for (int32_t w : gs.writers) {
+    int r = comm_rank_of(c, w);
+    if (r < 0) return fail(JITC_EINVAL, "jitc_restore: a writer is not in the communicator");
+    in.writers.push_back(r);
   }
-  std::vector<int> dst;  // comm ranks of members that are not writers
   for (int32_t m : gs.members) {
     if (std::find(gs.writers.begin(), gs.writers.end(), m) != gs.writers.end()) continue;
     int r = comm_rank_of(c, m);
-    if (r >= 0) dst.push_back(r);
+    if (r >= 0) in.dests.push_back(r);
   }
-  const int me = c->comm_rank;
-  int my_s = -1;
-  for (int s = 0; s < k; ++s)
-    if (wc[s] == me) my_s = s;
-  const bool is_dst = std::find(dst.begin(), dst.end(), me) != dst.end();
+  const int my_s = (int)(std::find(in.writers.begin(), in.writers.end(), in.me) - in.writers.begin());
+  const bool is_writer = my_s < (int)in.writers.size();
+  const bool is_dst = std::find(in.dests.begin(), in.dests.end(), in.me) != in.dests.end();
+  std::vector<PlanOp> ops;
+  uint32_t S = 0;
+  jitc_status st = make_plan(c, in, &ops, &S);
+  if (st) return st;
   // 1. the lowest writer broadcasts the expected digests (collective over the comm)
-  uint64_t* d_expect = g.d_dig;  // reuse the K1 buffer: holds d[] of the selected class
-  if (my_s == 0) {
+  uint64_t* d_expect = g.d_dig;
+  if (is_writer && my_s == 0) {
     if (!g.has_fp || g.fp_root != gs.root) return fail(JITC_ESTATE, "jitc_restore: writer fingerprint differs");
     CU(cudaMemcpyAsync(d_expect, g.fp.data(), g.n_c * 8, cudaMemcpyHostToDevice, c->s_comp));
   }
-  if (g.n_c) NC(ncclBroadcast(d_expect, d_expect, g.n_c, ncclUint64, wc[0], c->comm, c->s_comp));
+  if (g.n_c) NC(ncclBroadcast(d_expect, d_expect, g.n_c, ncclUint64, in.writers[0], c->comm, c->s_comp));
   std::vector<uint64_t> want(g.n_c);
   if (g.n_c) CU(cudaMemcpyAsync(want.data(), d_expect, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
   CU(cudaStreamSynchronize(c->s_comp));
   if (root_of(g.layout_hash, want.data(), g.n_c) != gs.root)
     return fail(JITC_ECORRUPT, "jitc_restore: broadcast digests do not chain to the selected root");
-  if (dst.empty() || (my_s < 0 && !is_dst)) return JITC_OK;
-  // 2. rounds: R bytes per writer per round, double-buffered
-  uint64_t per = std::max(k, 1);
-  uint64_t R = c->staging_bytes / (2ull * per) / g.C * g.C;
-  R = std::min<uint64_t>(R, c->slot_bytes);
-  if (R == 0) return fail(JITC_ENOMEM, "jitc_restore: staging too small for PEER rounds");
-  std::vector<uint64_t> q0(k), q1(k);
-  uint64_t maxlen = 0;
-  for (int s = 0; s < k; ++s) {
-    uint64_t c0, c1;
-    shard_range(g.n_c, k, s, &c0, &c1);
-    q0[s] = std::min(c0 * g.C, g.L);
-    q1[s] = std::min(c1 * g.C, g.L);
-    maxlen = std::max(maxlen, q1[s] - q0[s]);
-  }
-  if (is_dst && g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
-  if (my_s >= 0 && g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
-  uint32_t J = (uint32_t)((maxlen + R - 1) / R);
-  for (uint32_t j = 0; j < J; ++j) {
-    int sl = (int)(j % 2);
-    uint8_t* buf = c->staging + (uint64_t)sl * per * R;
-    jitc_status st;
-    if (my_s >= 0) {
-      uint64_t a = q0[my_s] + j * R, b = std::min(q1[my_s], a + R);
-      if (b > a) {
-        uint32_t lo, hi;
-        seg_span(g, a, b, &lo, &hi);
-        st = run_segments(c, g, kPack, one_range(lo, hi, buf, a), g.d_dig2, b - a);
-        if (st) return st;
-        NC(ncclGroupStart());
-        for (int d : dst) NC(ncclSend(buf, b - a, ncclUint8, d, c->comm, c->s_comp));
-        NC(ncclGroupEnd());
-        if (stats) stats->p2p_bytes += (b - a) * dst.size();
-      }
-    } else {
-      LaunchRanges lr{};
-      uint64_t bytes = 0;
-      NC(ncclGroupStart());
-      for (int s = 0; s < k; ++s) {
-        uint64_t a = q0[s] + j * R, b = std::min(q1[s], a + R);
-        if (b <= a) continue;
-        NC(ncclRecv(buf + s * R, b - a, ncclUint8, wc[s], c->comm, c->s_comp));
-      }
-      NC(ncclGroupEnd());
-      for (int s = 0; s < k; ++s) {
-        uint64_t a = q0[s] + j * R, b = std::min(q1[s], a + R);
-        if (b <= a) continue;
-        uint32_t lo, hi;
-        seg_span(g, a, b, &lo, &hi);
-        add_range(lr, lo, hi, buf + s * R, a);
-        bytes += b - a;
-        if (lr.n == kMaxRanges) {
-          st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
-          if (st) return st;
-          lr = LaunchRanges{};
-          bytes = 0;
-        }
-      }
-      if (lr.n) {
-        st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
-        if (st) return st;
-      }
-      if (stats) stats->p2p_bytes += bytes;
-    }
-  }
-  if (stats) stats->rounds += J;
+  if (!is_writer && !is_dst) return JITC_OK;
+  if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
+  // 2. data rounds
+  st = execute_plan(c, g, ops, S, stats);
+  if (st) return st;
   CU(cudaStreamSynchronize(c->s_comp));
   if (is_dst) {
-    jitc_status st = compare_digests(c, g, want, stats);
+    st = compare_digests(c, g, want, stats);
     if (st) return st;
     g.man_d = want;
     g.man_root = gs.root;
     g.has_man = true;
     if (stats) stats->image_bytes += g.L;
-  } else if (my_s >= 0 && g.n_c) {  // the writer's re-digest of its own range must still match
+  } else if (g.n_c) {  // the writer's re-digest of its own range must still match
     CU(cudaMemcpyAsync(c->h_dig, g.d_dig2, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
     CU(cudaStreamSynchronize(c->s_comp));
     uint64_t c0, c1;
-    shard_range(g.n_c, k, my_s, &c0, &c1);
+    shard_range(g.n_c, in.writers.size(), my_s, &c0, &c1);
     for (uint64_t ch = c0; ch < c1; ++ch)
       if (c->h_dig[ch] != want[ch]) return fail(JITC_EUNSTABLE, "jitc_restore: writer state changed");
   }

@@ -221,6 +221,43 @@ inline void shard_range(uint64_t n_c, uint64_t k, uint64_t s, uint64_t* c0, uint
   *c1 = ((s + 1) * n_c) / k;
 }
 uint64_t root_of(uint64_t layout_hash, const uint64_t* d, uint64_t n_c);
+
+// ------------------------------------------------------------------ restore plan (jitc_plan.cc)
+enum : uint8_t { kOpH2D = 1, kOpAllGather = 2, kOpPack = 3, kOpSend = 4, kOpRecv = 5, kOpUnpack = 6,
+                 kOpBcastDigests = 7 };
+constexpr uint32_t kMagicPlan = 0x5054494Au;      // "JITP"
+#pragma pack(push, 1)
+struct PlanOp {      // 48 B
+  uint32_t round;
+  uint8_t kind;
+  uint8_t slot;      // staging slot (double/multi-buffer index)
+  uint16_t pad;
+  int32_t peer;      // comm rank: H2D/PACK = self, SEND/RECV = the other side, UNPACK = block owner,
+                     // BCAST = root
+  uint32_t pad2;
+  uint64_t a, b;     // image byte range
+  uint64_t off;      // staging byte offset (ALLGATHER: base of the n blocks)
+  uint64_t bytes;    // bytes moved (ALLGATHER: block size R per rank)
+};
+struct PlanHdr {     // 24 B
+  uint32_t magic;
+  uint32_t n_ops;
+  uint64_t round_bytes;
+  uint32_t slots;
+  uint32_t pad;
+};
+#pragma pack(pop)
+static_assert(sizeof(PlanOp) == 48, "plan op");
+static_assert(sizeof(PlanHdr) == 24, "plan header");
+struct PlanInput {
+  int mode = 0;
+  uint64_t n_c = 0, chunk_bytes = 0, image_bytes = 0;
+  int n = 1, me = 0;                   // communicator size and this rank
+  std::vector<int32_t> writers, dests;  // comm ranks (PEER)
+  uint64_t staging_bytes = 0, slot_bytes = 0;
+};
+bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
+                        std::string* why);
 uint64_t manifest_trailer(const uint8_t* p, size_t n);
 
 // thread-local error text

@@ -1,0 +1,186 @@
+// Restore round schedule (pure host code).  jitc_restore executes exactly
+// this list of operations; jitc_restore_plan exports it so the multi-rank
+// logic can be checked without GPUs (tests/test_multirank_gloo.py).
+//
+// HOST (every rank restarts; reading R17): comm rank r loads
+// chunk range O5(n_c, n, r) of the committed image H2D; every round the ranks
+// all-gather R-byte blocks over NVLink (in place: rank q's block sits at
+// q*R); K3 unpacks every rank's block.
+// PEER (only the replacement lost its state): writer s packs
+// its O5(n_c, k, s) range from live HBM (K2) and sends it to every member
+// that is not a writer; receivers unpack all k blocks (K3).
+#include <string.h>
+
+#include <algorithm>
+
+#include "jitc_internal.h"
+
+namespace jitc {
+
+static void o5_bytes(uint64_t n_c, uint64_t k, uint64_t s, uint64_t C, uint64_t L, uint64_t* a, uint64_t* b) {
+  unsigned __int128 c0 = (unsigned __int128)s * n_c / k, c1 = (unsigned __int128)(s + 1) * n_c / k;
+  *a = std::min<uint64_t>((uint64_t)c0 * C, L);
+  *b = std::min<uint64_t>((uint64_t)c1 * C, L);
+}
+
+bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
+                        std::string* why) {
+  ops->clear();
+  const uint64_t C = in.chunk_bytes, L = in.image_bytes, n_c = in.n_c;
+  if (C == 0 || in.n <= 0 || in.me < 0 || in.me >= in.n) {
+    *why = "bad plan input";
+    return false;
+  }
+  if (in.mode == JITC_RESTORE_HOST) {
+    const uint64_t n = (uint64_t)in.n;
+    uint64_t R = std::min<uint64_t>(in.slot_bytes, in.staging_bytes / (2 * n)) / C * C;
+    if (R == 0) {
+      *why = "staging too small for the restore rounds (need >= 2 * n * C bytes)";
+      return false;
+    }
+    uint64_t S = std::max<uint64_t>(2, std::min<uint64_t>(8, in.staging_bytes / (n * R)));
+    *round_bytes = R;
+    *slots = (uint32_t)S;
+    std::vector<uint64_t> q0(n), q1(n);
+    uint64_t maxlen = 0;
+    for (uint64_t r = 0; r < n; ++r) {
+      o5_bytes(n_c, n, r, C, L, &q0[r], &q1[r]);
+      maxlen = std::max(maxlen, q1[r] - q0[r]);
+    }
+    const uint64_t J = (maxlen + R - 1) / R;
+    for (uint64_t j = 0; j < J; ++j) {
+      const uint32_t sl = (uint32_t)(j % S);
+      const uint64_t base = sl * n * R;
+      uint64_t a = q0[in.me] + j * R, b = std::min(q1[in.me], a + R);
+      if (b > a) ops->push_back(PlanOp{(uint32_t)j, kOpH2D, (uint8_t)sl, 0, in.me, 0, a, b, base + in.me * R, b - a});
+      if (n > 1) ops->push_back(PlanOp{(uint32_t)j, kOpAllGather, (uint8_t)sl, 0, -1, 0, 0, 0, base, R});
+      for (uint64_t q = 0; q < n; ++q) {
+        uint64_t qa = q0[q] + j * R, qb = std::min(q1[q], qa + R);
+        if (qb > qa) ops->push_back(PlanOp{(uint32_t)j, kOpUnpack, (uint8_t)sl, 0, (int32_t)q, 0, qa, qb, base + q * R, qb - qa});
+      }
+    }
+    return true;
+  }
+  if (in.mode != JITC_RESTORE_PEER) {
+    *why = "bad mode";
+    return false;
+  }
+  const uint64_t k = in.writers.size();
+  if (k == 0) {
+    *round_bytes = 0;
+    *slots = 0;
+    return true;  // dropped group: nothing moves
+  }
+  for (int32_t w : in.writers)
+    if (w < 0 || w >= in.n) {
+      *why = "a writer is not in the communicator";
+      return false;
+    }
+  uint64_t R = std::min<uint64_t>(in.slot_bytes, in.staging_bytes / (2 * k)) / C * C;
+  if (R == 0) {
+    *why = "staging too small for the PEER rounds (need >= 2 * k * C bytes)";
+    return false;
+  }
+  const uint64_t S = 2;
+  *round_bytes = R;
+  *slots = (uint32_t)S;
+  int my_s = -1;
+  for (uint64_t s = 0; s < k; ++s)
+    if (in.writers[s] == in.me) my_s = (int)s;
+  const bool is_dst = std::find(in.dests.begin(), in.dests.end(), in.me) != in.dests.end();
+  ops->push_back(PlanOp{0, kOpBcastDigests, 0, 0, in.writers[0], 0, 0, 0, 0, n_c * 8});
+  if (in.dests.empty() || (my_s < 0 && !is_dst)) return true;
+  std::vector<uint64_t> q0(k), q1(k);
+  uint64_t maxlen = 0;
+  for (uint64_t s = 0; s < k; ++s) {
+    o5_bytes(n_c, k, s, C, L, &q0[s], &q1[s]);
+    maxlen = std::max(maxlen, q1[s] - q0[s]);
+  }
+  const uint64_t J = (maxlen + R - 1) / R;
+  for (uint64_t j = 0; j < J; ++j) {
+    const uint32_t sl = (uint32_t)(j % S);
+    const uint64_t base = sl * k * R;
+    if (my_s >= 0) {
+      uint64_t a = q0[my_s] + j * R, b = std::min(q1[my_s], a + R);
+      if (b <= a) continue;
+      ops->push_back(PlanOp{(uint32_t)j, kOpPack, (uint8_t)sl, 0, in.me, 0, a, b, base, b - a});
+      for (int32_t d : in.dests) ops->push_back(PlanOp{(uint32_t)j, kOpSend, (uint8_t)sl, 0, d, 0, a, b, base, b - a});
+    } else {
+      for (uint64_t s = 0; s < k; ++s) {
+        uint64_t a = q0[s] + j * R, b = std::min(q1[s], a + R);
+        if (b > a) ops->push_back(PlanOp{(uint32_t)j, kOpRecv, (uint8_t)sl, 0, in.writers[s], 0, a, b, base + s * R, b - a});
+      }
+      for (uint64_t s = 0; s < k; ++s) {
+        uint64_t a = q0[s] + j * R, b = std::min(q1[s], a + R);
+        if (b > a) ops->push_back(PlanOp{(uint32_t)j, kOpUnpack, (uint8_t)sl, 0, in.writers[s], 0, a, b, base + s * R, b - a});
+      }
+    }
+  }
+  return true;
+}
+
+}  // namespace jitc
+
+using namespace jitc;
+
+extern "C" jitc_status jitc_restore_plan(const void* selection, size_t sel_len, uint32_t group, int32_t mode,
+                                         const int32_t* comm_job_ranks, int32_t n, int32_t comm_rank,
+                                         uint64_t staging_bytes, uint64_t slot_bytes, void* plan, size_t cap,
+                                         size_t* len) {
+  if (!selection || !comm_job_ranks || !len || n <= 0) {
+    set_error("jitc_restore_plan: bad argument");
+    return JITC_EINVAL;
+  }
+  Selection sel;
+  std::string why;
+  if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why)) {
+    set_error("jitc_restore_plan: " + why);
+    return JITC_EINVAL;
+  }
+  const GroupSelection* gs = sel.find(group);
+  if (!gs) {
+    set_error("jitc_restore_plan: group not in selection");
+    return JITC_EINVAL;
+  }
+  auto comm_of = [&](int32_t job) {
+    for (int i = 0; i < n; ++i)
+      if (comm_job_ranks[i] == job) return i;
+    return -1;
+  };
+  PlanInput in;
+  in.mode = mode;
+  in.n_c = gs->n_c;
+  in.chunk_bytes = gs->chunk_bytes;
+  in.image_bytes = gs->image_bytes;
+  in.n = n;
+  in.me = comm_rank;
+  in.staging_bytes = staging_bytes;
+  in.slot_bytes = slot_bytes;
+  for (int32_t w : gs->writers) in.writers.push_back(comm_of(w));
+  for (int32_t m : gs->members) {
+    if (std::find(gs->writers.begin(), gs->writers.end(), m) != gs->writers.end()) continue;
+    int r = comm_of(m);
+    if (r >= 0) in.dests.push_back(r);
+  }
+  std::vector<PlanOp> ops;
+  uint64_t R = 0;
+  uint32_t S = 0;
+  if (!build_restore_plan(in, &ops, &R, &S, &why)) {
+    set_error("jitc_restore_plan: " + why);
+    return JITC_EINVAL;
+  }
+  PlanHdr h{};
+  h.magic = kMagicPlan;
+  h.n_ops = (uint32_t)ops.size();
+  h.round_bytes = R;
+  h.slots = S;
+  *len = sizeof h + ops.size() * sizeof(PlanOp);
+  if (cap == 0) return JITC_OK;
+  if (cap < *len || !plan) {
+    set_error("jitc_restore_plan: buffer too small");
+    return JITC_EINVAL;
+  }
+  memcpy(plan, &h, sizeof h);
+  if (!ops.empty()) memcpy(static_cast<uint8_t*>(plan) + sizeof h, ops.data(), ops.size() * sizeof(PlanOp));
+  return JITC_OK;
+}

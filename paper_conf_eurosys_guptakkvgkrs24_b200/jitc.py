@@ -99,6 +99,7 @@ def lib() -> ctypes.CDLL:
         "jitc_verify": ([vp, u32, vp, sz, P(u64)], i32),
         "jitc_layout": ([P(Tensor), sz, u64, P(u64), P(u64), P(u64)], i32),
         "jitc_shard_range": ([u64, u32, u32, P(u64), P(u64)], i32),
+        "jitc_restore_plan": ([vp, sz, u32, i32, P(i32), i32, i32, u64, u64, vp, sz, P(sz)], i32),
         "jitc_kernel_counters": ([vp, i32, P(KernelCounter)], i32),
         "jitc_reset_counters": ([vp], i32),
         "jitc_gen_fill": ([vp, u32, u64, u64, u32, u32, u32, u32, i32, vp], i32),
@@ -118,7 +119,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_declare_group", "jitc_mark", "jitc_phase", "jitc_get_unique_id", "jitc_comm_init",
             "jitc_comm_shrink", "jitc_comm_destroy", "jitc_fingerprint", "jitc_exchange_records",
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
-            "jitc_layout", "jitc_shard_range", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
+            "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip"]
 
 
@@ -182,6 +183,28 @@ def parse_selection(sel: bytes) -> dict:
                                   excluded=[(ints[k + n_mem + 2 * j], ints[k + n_mem + 2 * j + 1]) for j in range(n_ex)],
                                   conflict_chunks=cf, layout_hash=lh, chunk_bytes=C, n_c=n_c, image_bytes=L, root=root))
     return out
+
+
+OP_NAMES = {1: "H2D", 2: "ALLGATHER", 3: "PACK", 4: "SEND", 5: "RECV", 6: "UNPACK", 7: "BCAST_DIGESTS"}
+
+
+def restore_plan(selection: bytes, group: int, mode: int, comm_job_ranks: Sequence[int], comm_rank: int,
+                 staging_bytes: int, slot_bytes: int) -> dict:
+    """The round schedule jitc_restore executes on `comm_rank` (pure; no GPU)."""
+    L = lib()
+    n = ctypes.c_size_t()
+    jr = _i32arr(list(comm_job_ranks))
+    args = (selection, len(selection), group, mode, jr, len(comm_job_ranks), comm_rank, staging_bytes, slot_bytes)
+    _check(L.jitc_restore_plan(*args, None, 0, ctypes.byref(n)), "jitc_restore_plan")
+    buf = ctypes.create_string_buffer(n.value)
+    _check(L.jitc_restore_plan(*args, buf, n.value, ctypes.byref(n)), "jitc_restore_plan")
+    raw = buf.raw[:n.value]
+    magic, n_ops, R, S, _ = struct.unpack_from("<IIQII", raw, 0)
+    ops = []
+    for i in range(n_ops):
+        rnd, kind, slot, _p, peer, _p2, a, b, off, nb = struct.unpack_from("<IBBHiIQQQQ", raw, 24 + 48 * i)
+        ops.append(dict(round=rnd, kind=OP_NAMES[kind], slot=slot, peer=peer, a=a, b=b, off=off, bytes=nb))
+    return dict(round_bytes=R, slots=S, ops=ops)
 
 
 def get_unique_id() -> bytes:
