@@ -100,6 +100,7 @@ struct jitc_ctx {
   int comm_n = 0, comm_rank = -1;
   std::vector<int32_t> comm_job;  // comm rank -> job rank
   uint64_t* d_small = nullptr;    // 64 B device scratch for size exchange / barrier
+  uint32_t* d_work = nullptr;     // K1/K2/K3 batch counters (self-resetting)
   uint64_t* h_small = nullptr;    // pinned
   // counters
   jitc_kernel_counter kc[4]{};
@@ -147,7 +148,7 @@ jitc_status run_segments(jitc_ctx* c, GroupState& g, int mode, const LaunchRange
                          uint64_t bytes) {
   bool timed = (c->cfg.flags & JITC_F_TIME_KERNELS) && c->kev_used + 2 <= c->kev.size();
   if (timed) CU(cudaEventRecord(c->kev[c->kev_used], c->s_comp));
-  CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->s_comp));
+  CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->d_work, c->s_comp));
   if (timed) {
     CU(cudaEventRecord(c->kev[c->kev_used + 1], c->s_comp));
     c->kev_kind[c->kev_used / 2] = mode;
@@ -353,6 +354,8 @@ jitc_status jitc_create(const jitc_config* cfg, jitc_ctx** out) {
   CU(cudaHostGetDevicePointer((void**)&c->phase_d, c->phase_h, 0));
   CU(cudaMalloc(&c->d_small, 64));
   CU(cudaMemset(c->d_small, 0, 64));
+  CU(cudaMalloc(&c->d_work, 64));
+  CU(cudaMemset(c->d_work, 0, 64));
   CU(cudaHostAlloc(&c->h_small, 64, cudaHostAllocDefault));
   void* fn = nullptr;
   cudaDriverEntryPointQueryResult q;
@@ -384,6 +387,7 @@ void jitc_destroy(jitc_ctx* c) {
   if (c->h_dig) cudaFreeHost(c->h_dig);
   if (c->h_small) cudaFreeHost(c->h_small);
   if (c->d_small) cudaFree(c->d_small);
+  if (c->d_work) cudaFree(c->d_work);
   if (c->own_staging && c->staging) cudaFree(c->staging);
   if (c->own_streams) {
     cudaStreamDestroy(c->s_comp);

@@ -69,8 +69,10 @@ struct LaunchRanges {
 };
 
 // kernels (jitc_kernels.cu)
+// d_work: 2 x u32 zero-initialised device counters, private to the stream
+// (the kernel resets them when it finishes).
 cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig,
-                            int grid, cudaStream_t s);
+                            int grid, uint32_t* d_work, cudaStream_t s);
 cudaError_t launch_phase_write(uint64_t* dev_slot, uint64_t value, cudaStream_t s);
 int segment_grid(int device);
 cudaError_t device_check(int device, std::string* why);

@@ -14,8 +14,8 @@
 // partial into d[chunk] with a 64-bit atomic and the result is deterministic.
 //
 // Work unit: one Seg = one piece (<= 32 KiB) of one tensor that never crosses
-// a chunk boundary.  Each CTA of a persistent grid takes an equal contiguous
-// run of segments; inside a segment every thread streams 16-byte vectors (4 loads in flight before
+// a chunk boundary.  CTAs of a persistent grid grab batches of 8 consecutive
+// segments from an atomic counter; inside a segment every thread streams 16-byte vectors (4 loads in flight before
 // any use), hashes both words, optionally stores, and the warp reduces its
 // partial with shuffles before one atomicAdd per warp per chunk it touched.  Pure HBM
 // (or PCIe) streaming: no tensor cores, no shared-memory reuse (every byte is
@@ -103,91 +103,113 @@ __device__ __forceinline__ void flush(unsigned long long* dig, uint32_t chunk, u
   if (lane == 0) atomicAdd(dig + chunk, (unsigned long long)acc);
 }
 
-// Every CTA takes a contiguous, equal-count run of segments (segments are
-// <= 32 KiB, so runs are balanced to within one segment), prefetches the
-// next descriptor while streaming the current one, and keeps the partial
-// digest in registers until the chunk changes.
+// Dynamic work distribution: CTAs grab batches of kBatch consecutive
+// segments (<= 256 KiB) from a global counter, so SMs that stream faster take
+// more work and no CTA idles at the tail.  Inside a batch the next
+// descriptor is prefetched while the current segment streams, and the
+// partial digest stays in registers until the chunk changes.  The counter
+// pair (next batch, finished CTAs) resets itself: the last CTA to finish
+// zeroes it for the next launch on the stream.
+constexpr uint32_t kBatch = 8;
+
 template <int MODE>
 __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ segs, LaunchRanges R,
-                                                       unsigned long long* __restrict__ dig) {
+                                                       unsigned long long* __restrict__ dig,
+                                                       unsigned int* __restrict__ work) {
   const uint32_t total = R.prefix[R.n];
-  const uint32_t v0 = (uint32_t)((uint64_t)blockIdx.x * total / gridDim.x);
-  const uint32_t v1 = (uint32_t)((uint64_t)(blockIdx.x + 1) * total / gridDim.x);
-  if (v0 >= v1) return;
+  const uint32_t nbatch = (total + kBatch - 1) / kBatch;
   const int tid = threadIdx.x;
   const int lane = tid & 31;
+  __shared__ uint32_t s_batch;
   uint64_t acc = 0;
-  int r;
-  Seg next = *seg_at(segs, R, v0, &r);
-  int next_r = r;
-  uint32_t cur_chunk = next.chunk;
-  for (uint32_t v = v0; v < v1; ++v) {
-    const Seg sg = next;
-    r = next_r;
-    if (v + 1 < v1) next = *seg_at(segs, R, v + 1, &next_r);
-    if (sg.chunk != cur_chunk) {
-      flush(dig, cur_chunk, acc, lane);
-      acc = 0;
-      cur_chunk = sg.chunk;
-    }
-    const uint64_t rel = sg.img_off - R.base_off[r];
-    uint8_t* img = reinterpret_cast<uint8_t*>(R.base[r]) + rel;  // 16-B aligned (staging / host image)
-    uint8_t* ten = reinterpret_cast<uint8_t*>(sg.src);
-    const uint64_t data = sg.data_bytes;
-    const uint64_t words = (data + sg.pad_bytes) >> 3;
-    const uint64_t g0 = sg.img_off >> 3;
-    uint64_t body_words = 0;
+  uint32_t cur_chunk = 0xFFFFFFFFu;
+  for (;;) {
+    if (tid == 0) s_batch = atomicAdd(work, 1u);
+    __syncthreads();
+    const uint32_t bidx = s_batch;
+    __syncthreads();
+    if (bidx >= nbatch) break;
+    const uint32_t v0 = bidx * kBatch, v1 = min(total, v0 + kBatch);
+    int r;
+    Seg next = *seg_at(segs, R, v0, &r);
+    int next_r = r;
+    for (uint32_t v = v0; v < v1; ++v) {
+      const Seg sg = next;
+      r = next_r;
+      if (v + 1 < v1) next = *seg_at(segs, R, v + 1, &next_r);
+      if (sg.chunk != cur_chunk) {
+        if (cur_chunk != 0xFFFFFFFFu) flush(dig, cur_chunk, acc, lane);
+        acc = 0;
+        cur_chunk = sg.chunk;
+      }
+      const uint64_t rel = sg.img_off - R.base_off[r];
+      uint8_t* img = reinterpret_cast<uint8_t*>(R.base[r]) + rel;  // 16-B aligned (staging / host image)
+      uint8_t* ten = reinterpret_cast<uint8_t*>(sg.src);
+      const uint64_t data = sg.data_bytes;
+      const uint64_t words = (data + sg.pad_bytes) >> 3;
+      const uint64_t g0 = sg.img_off >> 3;
+      uint64_t body_words = 0;
 
-    if (sg.flags & kSegAligned16) {
-      const uint32_t nvec = (uint32_t)(data >> 4);
-      body_words = 2ull * nvec;
-      const uint4* in = MODE == kUnpack ? reinterpret_cast<const uint4*>(img)
-                                        : reinterpret_cast<const uint4*>(ten);
-      uint4* out = MODE == kPack ? reinterpret_cast<uint4*>(img)
-                 : MODE == kUnpack ? reinterpret_cast<uint4*>(ten) : nullptr;
-      uint32_t i = tid;
-      // key of word 2i is (g0 + 2i + 1) * PHI; the step between a thread's
-      // consecutive vectors is 2 * kThreads words.
-      uint64_t key = (g0 + 2ull * i + 1ull) * PHI;
-      const uint64_t kstep = 2ull * kThreads * PHI;
-      for (; i + (kUnroll - 1) * kThreads < nvec; i += kUnroll * kThreads) {
-        uint4 x[kUnroll];
+      if (sg.flags & kSegAligned16) {
+        const uint32_t nvec = (uint32_t)(data >> 4);
+        body_words = 2ull * nvec;
+        const uint4* in = MODE == kUnpack ? reinterpret_cast<const uint4*>(img)
+                                          : reinterpret_cast<const uint4*>(ten);
+        uint4* out = MODE == kPack ? reinterpret_cast<uint4*>(img)
+                   : MODE == kUnpack ? reinterpret_cast<uint4*>(ten) : nullptr;
+        uint32_t i = tid;
+        // key of word 2i is (g0 + 2i + 1) * PHI; the step between a thread's
+        // consecutive vectors is 2 * kThreads words.
+        uint64_t key = (g0 + 2ull * i + 1ull) * PHI;
+        const uint64_t kstep = 2ull * kThreads * PHI;
+        for (; i + (kUnroll - 1) * kThreads < nvec; i += kUnroll * kThreads) {
+          uint4 x[kUnroll];
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) x[u] = MODE == kUnpack ? ld_plain(in + i + u * kThreads)
-                                                                 : ld_stream(in + i + u * kThreads);
+          for (int u = 0; u < kUnroll; ++u) x[u] = MODE == kUnpack ? ld_plain(in + i + u * kThreads)
+                                                                   : ld_stream(in + i + u * kThreads);
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
-          acc += dmix(lo64(x[u]) ^ key);
-          acc += dmix(hi64(x[u]) ^ (key + PHI));
+          for (int u = 0; u < kUnroll; ++u) {
+            acc += dmix(lo64(x[u]) ^ key);
+            acc += dmix(hi64(x[u]) ^ (key + PHI));
+            key += kstep;
+            if (MODE != kDigest) st_stream(out + i + u * kThreads, x[u]);
+          }
+        }
+        for (; i < nvec; i += kThreads) {
+          uint4 x = MODE == kUnpack ? ld_plain(in + i) : ld_stream(in + i);
+          acc += dmix(lo64(x) ^ key);
+          acc += dmix(hi64(x) ^ (key + PHI));
           key += kstep;
-          if (MODE != kDigest) st_stream(out + i + u * kThreads, x[u]);
+          if (MODE != kDigest) st_stream(out + i, x);
         }
       }
-      for (; i < nvec; i += kThreads) {
-        uint4 x = MODE == kUnpack ? ld_plain(in + i) : ld_stream(in + i);
-        acc += dmix(lo64(x) ^ key);
-        acc += dmix(hi64(x) ^ (key + PHI));
-        key += kstep;
-        if (MODE != kDigest) st_stream(out + i, x);
+      // Remaining words: unaligned tensors (all of them), the < 16-byte data
+      // tail, and the zero padding that closes the tensor's image slot.
+      const bool al8 = (sg.flags & kSegAligned8) != 0;
+      for (uint64_t w = body_words + tid; w < words; w += kThreads) {
+        const uint64_t b = 8 * w;
+        uint64_t x;
+        if (MODE == kUnpack) {
+          x = *reinterpret_cast<const uint64_t*>(img + b);
+          if (b < data) store_word_bytes(ten, b, data, x, al8);
+        } else {
+          x = load_word_bytes(ten, b, data, al8);
+          if (MODE == kPack) *reinterpret_cast<uint64_t*>(img + b) = x;
+        }
+        acc += dmix(x ^ ((g0 + w + 1ull) * PHI));
       }
-    }
-    // Remaining words: unaligned tensors (all of them), the < 16-byte data
-    // tail, and the zero padding that closes the tensor's image slot.
-    const bool al8 = (sg.flags & kSegAligned8) != 0;
-    for (uint64_t w = body_words + tid; w < words; w += kThreads) {
-      const uint64_t b = 8 * w;
-      uint64_t x;
-      if (MODE == kUnpack) {
-        x = *reinterpret_cast<const uint64_t*>(img + b);
-        if (b < data) store_word_bytes(ten, b, data, x, al8);
-      } else {
-        x = load_word_bytes(ten, b, data, al8);
-        if (MODE == kPack) *reinterpret_cast<uint64_t*>(img + b) = x;
-      }
-      acc += dmix(x ^ ((g0 + w + 1ull) * PHI));
     }
   }
-  flush(dig, cur_chunk, acc, lane);
+  if (cur_chunk != 0xFFFFFFFFu) flush(dig, cur_chunk, acc, lane);
+  // the last CTA out resets the counters for the next launch on this stream
+  if (tid == 0) {
+    __threadfence();
+    if (atomicAdd(work + 1, 1u) == gridDim.x - 1) {
+      work[0] = 0;
+      work[1] = 0;
+      __threadfence();
+    }
+  }
 }
 
 __global__ void phase_write_kernel(volatile uint64_t* slot, uint64_t value) {
@@ -291,15 +313,16 @@ cudaError_t device_check(int device, std::string* why) {
 }
 
 cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig, int grid,
-                            cudaStream_t s) {
+                            uint32_t* d_work, cudaStream_t s) {
   uint32_t total = r.prefix[r.n];
   if (total == 0) return cudaSuccess;
-  int g = (int)(total < (uint32_t)grid ? total : (uint32_t)grid);
+  uint32_t nbatch = (total + kBatch - 1) / kBatch;
+  int g = (int)(nbatch < (uint32_t)grid ? nbatch : (uint32_t)grid);
   auto* dig = reinterpret_cast<unsigned long long*>(d_dig);
   switch (mode) {
-    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig); break;
-    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig); break;
-    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig); break;
+    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work); break;
+    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work); break;
+    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();

@@ -61,6 +61,9 @@ int main(int argc, char** argv) {
   uint8_t* host;
   CK(cudaHostAlloc(&host, 4ull << 30, cudaHostAllocDefault));
   int grid = segment_grid(0);
+  uint32_t* work;
+  CK(cudaMalloc(&work, 64));
+  CK(cudaMemset(work, 0, 64));
   uint32_t per = (uint32_t)(launch_bytes / seg_bytes);
   uint32_t nl = (uint32_t)(arena_bytes / launch_bytes);
   std::vector<cudaEvent_t> ev(2 * nl + 2);
@@ -78,7 +81,7 @@ int main(int argc, char** argv) {
       r.base[0] = (uint64_t)stage;
       r.base_off[0] = (uint64_t)base * seg_bytes;
       if (each) CK(cudaEventRecord(ev[2 + 2 * j], s));
-      CK(launch_segments(mode, d_segs, r, dig, grid, s));
+      CK(launch_segments(mode, d_segs, r, dig, grid, work, s));
       if (each) CK(cudaEventRecord(ev[3 + 2 * j], s));
     }
     CK(cudaEventRecord(ev[1], s));
