@@ -292,7 +292,7 @@ def run_jitc(args):
                        "writers_k": world, "restore_mode": "HOST", "image": "shared /dev/shm",
                        "zero_copy": bool(args.zero_copy), "chunk_bytes": 1 << 20,
                        "staging_mib": args.staging, "slot_mib": args.slot,
-                       "l2": "state 24.9 GB >> 126 MB L2; no flush needed", "setup_s": round(setup_s, 1)},
+                       "l2": f"state {L_total / 1e9:.1f} GB >> 126 MB L2; no flush needed", "setup_s": round(setup_s, 1)},
             "seconds_to_recover": round(ms_step * 1e-3, 4),
             "phases_ms_median": med,
             "capture_GBps": round(L_total / world / (cap_ms * 1e-3) / 1e9, 3),
