@@ -266,6 +266,29 @@ jitc_status jitc_restore_plan(const void* selection, size_t sel_len, uint32_t gr
                               uint64_t staging_bytes, uint64_t slot_bytes, void* plan, size_t cap,
                               size_t* len);
 
+/* ---- hang detection (NEXT-1; §3.1-3.2) ------------------ */
+/* The caller records a CUDA event after each collective on its NCCL stream
+ * (the event the compute stream waits on, PAPER.md:122 / Fig. 3) and puts it
+ * on the watch-list; completed events drop off.  A native watchdog thread
+ * polls the list with cudaEventQuery every 200 us; an event still incomplete
+ * `timeout_ms` after it was added is a hang.  On a hang the watchdog thread
+ * runs the action itself -- JITC_ON_HANG_LOCAL_CAPTURE: fingerprint, select
+ * over this rank's own record, capture, commit (no collective; the paper's
+ * user-level protocol), entirely in C++ on the library's
+ * non-blocking streams, so neither the GIL nor the blocked default stream can
+ * stop it -- then calls fn(user, tag, waited_ms) if given,
+ * and stops.  While the watchdog runs, other threads may call only
+ * jitc_watch_event / jitc_watchdog_wait / jitc_watchdog_stop on the ctx. */
+typedef void (*jitc_hang_fn)(void* user, uint64_t tag, double waited_ms);
+enum { JITC_ON_HANG_NOTIFY = 0, JITC_ON_HANG_LOCAL_CAPTURE = 1 };
+jitc_status jitc_watch_event(jitc_ctx* ctx, void* event, uint64_t tag);
+jitc_status jitc_watchdog_start(jitc_ctx* ctx, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user);
+/* Blocks up to max_ms for the hang action to finish.  *fired = 1 if it did;
+ * returns the action's status (JITC_OK when nothing fired). */
+jitc_status jitc_watchdog_wait(jitc_ctx* ctx, uint32_t max_ms, int32_t* fired, uint64_t* tag, double* waited_ms,
+                               double* action_ms, jitc_stats* action_stats);
+jitc_status jitc_watchdog_stop(jitc_ctx* ctx);
+
 /* ---- counters ---------------------------------------------------------------- */
 jitc_status jitc_kernel_counters(jitc_ctx* ctx, int32_t kind, jitc_kernel_counter* out);
 jitc_status jitc_reset_counters(jitc_ctx* ctx);
@@ -285,6 +308,12 @@ jitc_status jitc_inject_update(void* dptr, uint64_t e0, uint64_t count, uint32_t
 jitc_status jitc_inject_rne(const void* master_f32, void* param_bf16, uint64_t count, void* stream);
 /* Flips bit `bit` of byte `byte` of device memory at dptr. */
 jitc_status jitc_inject_bitflip(void* dptr, uint64_t byte, uint32_t bit, void* stream);
+/* Emulates a collective hung on a failed peer: launches
+ * n_ctas spinning CTAs on `stream` that wait on device flag `slot` (0..63),
+ * as NCCL kernels wait on flags their peers write; jitc_inject_release(slot)
+ * sets the flag from a kernel on a separate stream and lets them exit. */
+jitc_status jitc_inject_hang(void* stream, int32_t n_ctas, uint32_t slot);
+jitc_status jitc_inject_release(uint32_t slot);
 
 #ifdef __cplusplus
 }

@@ -20,6 +20,9 @@
 
 #include <algorithm>
 #include <chrono>
+#include <condition_variable>
+#include <mutex>
+#include <thread>
 #include <map>
 #include <memory>
 #include <string>
@@ -102,6 +105,25 @@ struct jitc_ctx {
   uint64_t* d_small = nullptr;    // 64 B device scratch for size exchange / barrier
   uint32_t* d_work = nullptr;     // K1/K2/K3 batch counters (self-resetting)
   uint64_t* h_small = nullptr;    // pinned
+  // watchdog (NEXT-1): explicit event watch-list polled by a native thread
+  struct Watch {
+    cudaEvent_t ev;
+    uint64_t tag;
+    double t_added;
+  };
+  std::mutex wmu;
+  std::condition_variable wcv;
+  std::vector<Watch> watches;
+  std::thread wthread;
+  bool wrun = false, fired = false, action_done = false;
+  uint64_t fired_tag = 0;
+  double detect_ms = 0, waited_ms = 0, action_ms = 0;
+  uint32_t timeout_ms = 0;
+  int action = 0;
+  jitc_hang_fn hang_fn = nullptr;
+  void* hang_user = nullptr;
+  jitc_status action_status = JITC_OK;
+  jitc_stats action_stats{};
   // counters
   jitc_kernel_counter kc[4]{};
   uint64_t launches_in_call = 0;
@@ -370,6 +392,7 @@ jitc_status jitc_create(const jitc_config* cfg, jitc_ctx** out) {
 
 void jitc_destroy(jitc_ctx* c) {
   if (!c) return;
+  jitc_watchdog_stop(c);
   cudaSetDevice(c->device);
   if (c->s_comp) cudaStreamSynchronize(c->s_comp);
   if (c->s_copy) cudaStreamSynchronize(c->s_copy);
@@ -846,7 +869,7 @@ static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelec
   return b;
 }
 
-jitc_status jitc_commit(jitc_ctx* c, const void* selection, size_t sel_len) {
+static jitc_status commit_impl(jitc_ctx* c, const void* selection, size_t sel_len, bool collective) {
   if (!c) return fail(JITC_EINVAL, "jitc_commit: null ctx");
   Selection sel;
   std::string why;
@@ -854,7 +877,7 @@ jitc_status jitc_commit(jitc_ctx* c, const void* selection, size_t sel_len) {
     return fail(JITC_EINVAL, "jitc_commit: " + why);
   if (sel.status != JITC_OK) return fail(sel.status, "jitc_commit: selection status is not OK");
   CU(cudaSetDevice(c->device));
-  jitc_status st = barrier(c);  // every writer's capture has returned
+  jitc_status st = collective ? barrier(c) : JITC_OK;  // every writer's capture has returned
   if (st) return st;
   for (auto& kv : c->groups) {
     GroupState& g = kv.second;
@@ -883,7 +906,11 @@ jitc_status jitc_commit(jitc_ctx* c, const void* selection, size_t sel_len) {
         return fail(JITC_EIO, "jitc_commit: writing commit record: " + std::string(strerror(errno)));
     }
   }
-  return barrier(c);  // nobody restores before every commit record exists
+  return collective ? barrier(c) : JITC_OK;  // nobody restores before every commit record exists
+}
+
+jitc_status jitc_commit(jitc_ctx* c, const void* selection, size_t sel_len) {
+  return commit_impl(c, selection, sel_len, true);
 }
 
 // ------------------------------------------------------------ restore
@@ -1235,6 +1262,137 @@ jitc_status jitc_verify(jitc_ctx* c, uint32_t group, const void* expected, size_
       if (first_bad) *first_bad = ch;
       return fail(JITC_ECORRUPT, "jitc_verify: chunk " + std::to_string(ch) + " differs");
     }
+  return JITC_OK;
+}
+
+// ------------------------------------------------------------ watchdog (NEXT-1)
+// PAPER.md:124-126 §3.1: events recorded after collectives are put on a
+// watch-list; a watchdog thread polls them with cudaEventQuery and treats
+// one that stays incomplete past a timeout as a hang of the collective.
+// PAPER.md:132-134 §3.2: the checkpoint is then taken on a side stream by the
+// watchdog thread itself -- here entirely in C++ (no Python callback, so the
+// GIL cannot block it) on the library's non-blocking streams.
+static jitc_status local_capture(jitc_ctx* c, jitc_stats* st) {
+  size_t len = 0;
+  jitc_status r = jitc_fingerprint(c, JITC_ALL_GROUPS, nullptr, 0, &len);
+  if (r) return r;
+  std::vector<uint8_t> blob(len);
+  r = jitc_fingerprint(c, JITC_ALL_GROUPS, blob.data(), blob.size(), &len);
+  if (r) return r;
+  int32_t me = c->cfg.rank;
+  size_t sl = 0;
+  jitc_select_consistent_replica(blob.data(), len, &me, 1, nullptr, 0, &sl);
+  std::vector<uint8_t> sel(sl);
+  r = jitc_select_consistent_replica(blob.data(), len, &me, 1, sel.data(), sel.size(), &sl);
+  if (r) return r;
+  r = jitc_capture(c, sel.data(), sl, JITC_ALL_GROUPS, st);
+  if (r) return r;
+  return commit_impl(c, sel.data(), sl, false);
+}
+
+static void watchdog_loop(jitc_ctx* c) {
+  cudaSetDevice(c->device);
+  const double t0 = now_ms();
+  for (;;) {
+    std::unique_lock<std::mutex> lk(c->wmu);
+    if (!c->wrun) return;
+    double now = now_ms();
+    bool hang = false;
+    for (size_t i = 0; i < c->watches.size();) {
+      cudaError_t q = cudaEventQuery(c->watches[i].ev);
+      if (q == cudaSuccess) {
+        c->watches.erase(c->watches.begin() + i);
+        continue;
+      }
+      if (q != cudaErrorNotReady) cudaGetLastError();
+      if (now - c->watches[i].t_added >= c->timeout_ms) {
+        hang = true;
+        c->fired_tag = c->watches[i].tag;
+        c->waited_ms = now - c->watches[i].t_added;
+        break;
+      }
+      ++i;
+    }
+    if (hang) {
+      c->fired = true;
+      c->detect_ms = now - t0;
+      lk.unlock();
+      double ta = now_ms();
+      if (c->action == JITC_ON_HANG_LOCAL_CAPTURE) {
+        jitc_stats st{};
+        jitc_status r = local_capture(c, &st);
+        lk.lock();
+        c->action_status = r;
+        c->action_stats = st;
+        lk.unlock();
+      }
+      if (c->hang_fn) c->hang_fn(c->hang_user, c->fired_tag, c->waited_ms);
+      lk.lock();
+      c->action_ms = now_ms() - ta;
+      c->action_done = true;
+      c->wrun = false;
+      c->wcv.notify_all();
+      return;
+    }
+    c->wcv.wait_for(lk, std::chrono::microseconds(200));
+  }
+}
+
+static void stop_thread(jitc_ctx* c) {
+  {
+    std::lock_guard<std::mutex> lk(c->wmu);
+    c->wrun = false;
+    c->wcv.notify_all();
+  }
+  if (c->wthread.joinable()) c->wthread.join();
+}
+
+jitc_status jitc_watch_event(jitc_ctx* c, void* event, uint64_t tag) {
+  if (!c || !event) return fail(JITC_EINVAL, "jitc_watch_event: null argument");
+  std::lock_guard<std::mutex> lk(c->wmu);
+  c->watches.push_back({(cudaEvent_t)event, tag, now_ms()});
+  return JITC_OK;
+}
+
+jitc_status jitc_watchdog_start(jitc_ctx* c, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user) {
+  if (!c) return fail(JITC_EINVAL, "jitc_watchdog_start: null ctx");
+  if (action != JITC_ON_HANG_NOTIFY && action != JITC_ON_HANG_LOCAL_CAPTURE)
+    return fail(JITC_EINVAL, "jitc_watchdog_start: bad action");
+  stop_thread(c);  // a previous watchdog; the watch-list is kept
+  std::lock_guard<std::mutex> lk(c->wmu);
+  c->timeout_ms = timeout_ms;
+  c->action = action;
+  c->hang_fn = fn;
+  c->hang_user = user;
+  c->fired = c->action_done = false;
+  c->action_status = JITC_OK;
+  c->action_stats = jitc_stats{};
+  c->action_stats.first_bad_chunk = -1;
+  c->wrun = true;
+  c->wthread = std::thread(watchdog_loop, c);
+  return JITC_OK;
+}
+
+jitc_status jitc_watchdog_wait(jitc_ctx* c, uint32_t max_ms, int32_t* fired, uint64_t* tag, double* waited_ms,
+                               double* action_ms, jitc_stats* action_stats) {
+  if (!c || !fired) return fail(JITC_EINVAL, "jitc_watchdog_wait: null argument");
+  std::unique_lock<std::mutex> lk(c->wmu);
+  c->wcv.wait_for(lk, std::chrono::milliseconds(max_ms), [c] { return c->action_done; });
+  *fired = c->action_done ? 1 : 0;
+  if (tag) *tag = c->fired_tag;
+  if (waited_ms) *waited_ms = c->waited_ms;
+  if (action_ms) *action_ms = c->action_ms;
+  if (action_stats) *action_stats = c->action_stats;
+  jitc_status st = c->action_done ? c->action_status : JITC_OK;
+  if (st) set_error("jitc_watchdog_wait: the on-hang capture failed with status " + std::to_string(st));
+  return st;
+}
+
+jitc_status jitc_watchdog_stop(jitc_ctx* c) {
+  if (!c) return fail(JITC_EINVAL, "jitc_watchdog_stop: null ctx");
+  stop_thread(c);
+  std::lock_guard<std::mutex> lk(c->wmu);
+  c->watches.clear();
   return JITC_OK;
 }
 

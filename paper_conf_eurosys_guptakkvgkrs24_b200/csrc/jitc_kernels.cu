@@ -24,6 +24,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <string.h>
+
 #include <string>
 
 #include "jitc_internal.h"
@@ -278,6 +280,22 @@ __global__ void rne_kernel(const uint32_t* m, uint16_t* p, uint64_t count) {
 
 __global__ void bitflip_kernel(uint8_t* p, uint8_t mask) { *p ^= mask; }
 
+// Emulated hung collective: spins on a DEVICE-memory flag (as NCCL kernels
+// spin on flags their peers write over NVLink), released by release_kernel
+// launched on a separate non-blocking stream.
+__global__ void hang_kernel(volatile uint32_t* flag) {
+  if (threadIdx.x == 0)
+    while (*flag == 0) __nanosleep(2000);
+  __syncthreads();
+}
+__global__ void release_kernel(uint32_t* flag, uint32_t v) {
+  *reinterpret_cast<volatile uint32_t*>(flag) = v;
+  __threadfence_system();
+}
+
+uint32_t* g_hang_d = nullptr;  // 64 device release flags
+cudaStream_t g_hang_s = nullptr;
+
 int g_grid[64] = {0};
 
 }  // namespace
@@ -294,6 +312,24 @@ int segment_grid(int device) {
   return g_grid[device];
 }
 
+// Force-load every kernel of this module.  With CUDA lazy loading
+// (CUDA_MODULE_LOADING=LAZY, the default) a kernel's first launch loads its
+// code, and that load waits behind work already running on the device -- e.g.
+// a collective hung on a dead peer -- so a first launch inside the failure
+// path would deadlock (measured: tools/wd_debug*.py).  jitc_create calls this.
+cudaError_t preload_kernels() {
+  cudaFuncAttributes fa;
+  const void* fns[] = {(const void*)seg_kernel<kDigest>, (const void*)seg_kernel<kPack>,
+                       (const void*)seg_kernel<kUnpack>, (const void*)phase_write_kernel,
+                       (const void*)gen_kernel, (const void*)update_kernel, (const void*)rne_kernel,
+                       (const void*)bitflip_kernel, (const void*)hang_kernel, (const void*)release_kernel};
+  for (const void* f : fns) {
+    cudaError_t e = cudaFuncGetAttributes(&fa, f);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
 cudaError_t device_check(int device, std::string* why) {
   cudaDeviceProp p;
   cudaError_t e = cudaGetDeviceProperties(&p, device);
@@ -306,8 +342,7 @@ cudaError_t device_check(int device, std::string* why) {
            "; libjitc is built for sm_100a only";
     return cudaErrorNoKernelImageForDevice;
   }
-  cudaFuncAttributes fa;
-  e = cudaFuncGetAttributes(&fa, seg_kernel<kDigest>);
+  e = preload_kernels();
   if (e != cudaSuccess) *why = std::string("sm_100a kernels not loadable: ") + cudaGetErrorString(e);
   return e;
 }
@@ -379,6 +414,30 @@ jitc_status jitc_inject_bitflip(void* dptr, uint64_t byte, uint32_t bit, void* s
   bitflip_kernel<<<1, 1, 0, (cudaStream_t)stream>>>((uint8_t*)dptr + byte, (uint8_t)(1u << bit));
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) { set_error(std::string("jitc_inject_bitflip: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
+  return JITC_OK;
+}
+
+jitc_status jitc_inject_hang(void* stream, int32_t n_ctas, uint32_t slot) {
+  if (n_ctas <= 0 || slot >= 64) { set_error("jitc_inject_hang: bad argument"); return JITC_EINVAL; }
+  cudaError_t e = cudaSuccess;
+  if (!g_hang_d) {
+    e = cudaMalloc(&g_hang_d, 64 * sizeof(uint32_t));
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&g_hang_s, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaMemset(g_hang_d, 0, 64 * sizeof(uint32_t));
+    if (e != cudaSuccess) { set_error(std::string("jitc_inject_hang: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
+  }
+  release_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(g_hang_d + slot, 0u);   // arm, in stream order
+  hang_kernel<<<n_ctas, 32, 0, (cudaStream_t)stream>>>(g_hang_d + slot);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) { set_error(std::string("jitc_inject_hang: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
+  return JITC_OK;
+}
+
+jitc_status jitc_inject_release(uint32_t slot) {
+  if (!g_hang_d || slot >= 64) { set_error("jitc_inject_release: no hang injected"); return JITC_EINVAL; }
+  release_kernel<<<1, 1, 0, g_hang_s>>>(g_hang_d + slot, 1u);
+  cudaError_t e = cudaStreamSynchronize(g_hang_s);
+  if (e != cudaSuccess) { set_error(std::string("jitc_inject_release: ") + cudaGetErrorString(e)); return JITC_ECUDA; }
   return JITC_OK;
 }
 

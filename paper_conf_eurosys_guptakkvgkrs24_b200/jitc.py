@@ -106,6 +106,12 @@ def lib() -> ctypes.CDLL:
         "jitc_inject_update": ([vp, u64, u64, u32, u64, vp], i32),
         "jitc_inject_rne": ([vp, vp, u64, vp], i32),
         "jitc_inject_bitflip": ([vp, u64, u32, vp], i32),
+        "jitc_inject_hang": ([vp, i32, u32], i32),
+        "jitc_inject_release": ([u32], i32),
+        "jitc_watch_event": ([vp, vp, u64], i32),
+        "jitc_watchdog_start": ([vp, u32, i32, vp, vp], i32),
+        "jitc_watchdog_wait": ([vp, u32, P(i32), P(u64), P(ctypes.c_double), P(ctypes.c_double), P(Stats)], i32),
+        "jitc_watchdog_stop": ([vp], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -120,7 +126,10 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_comm_shrink", "jitc_comm_destroy", "jitc_fingerprint", "jitc_exchange_records",
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
-            "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip"]
+            "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
+            "jitc_inject_release", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
+            "jitc_watchdog_stop"]
+ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE = 0, 1
 
 
 def last_error() -> str:
@@ -232,6 +241,15 @@ def inject_bitflip(ptr: int, byte: int, bit: int, stream: int = 0):
     _check(lib().jitc_inject_bitflip(ptr, byte, bit, stream or None), "jitc_inject_bitflip")
 
 
+def inject_hang(stream: int, n_ctas: int, slot: int = 0):
+    """Spinning CTAs on `stream` that emulate a collective hung on a dead peer."""
+    _check(lib().jitc_inject_hang(stream or None, n_ctas, slot), "jitc_inject_hang")
+
+
+def inject_release(slot: int = 0):
+    _check(lib().jitc_inject_release(slot), "jitc_inject_release")
+
+
 # ------------------------------------------------------------------ context
 class Context:
     """One libjitc context (one GPU, one process).  Methods map 1:1 to the C ABI."""
@@ -336,6 +354,33 @@ class Context:
         r = self._L.jitc_verify(self._h, group, expected, len(expected) if expected else 0, ctypes.byref(fb))
         _check(r, "jitc_verify", fb.value if r == ECORRUPT else -1)
         return fb.value
+
+    # -- hang detection (NEXT-1)
+    def watch_event(self, event_handle: int, tag: int):
+        _check(self._L.jitc_watch_event(self._h, event_handle, tag), "jitc_watch_event")
+
+    def watchdog_start(self, timeout_ms: int, action: int = ON_HANG_NOTIFY):
+        _check(self._L.jitc_watchdog_start(self._h, timeout_ms, action, None, None), "jitc_watchdog_start")
+
+    def watchdog_wait(self, max_ms: int, hold_gil: bool = False) -> dict:
+        """Blocks until the on-hang action finished (or max_ms).  hold_gil=True
+        calls through ctypes.PyDLL, i.e. WITHOUT releasing the GIL, to show the
+        capture needs no Python thread."""
+        f = ctypes.PyDLL(SO_PATH).jitc_watchdog_wait if hold_gil else self._L.jitc_watchdog_wait
+        if hold_gil:
+            f.argtypes = self._L.jitc_watchdog_wait.argtypes
+            f.restype = ctypes.c_int32
+        fired, tag = ctypes.c_int32(), ctypes.c_uint64()
+        waited, act = ctypes.c_double(), ctypes.c_double()
+        st = Stats()
+        r = f(self._h, max_ms, ctypes.byref(fired), ctypes.byref(tag), ctypes.byref(waited), ctypes.byref(act),
+              ctypes.byref(st))
+        _check(r, "jitc_watchdog_wait")
+        return dict(fired=bool(fired.value), tag=tag.value, waited_ms=waited.value, action_ms=act.value,
+                    stats=st.as_dict())
+
+    def watchdog_stop(self):
+        _check(self._L.jitc_watchdog_stop(self._h), "jitc_watchdog_stop")
 
     def kernel_counters(self, kind: int) -> dict:
         kc = KernelCounter()

@@ -42,6 +42,8 @@ class GroupState:
         for t, p in zip(self.spec.tensors, self.ptrs):
             lo, hi, pos = t.range
             jitc.gen_fill(p, DTYPE_CODE[t.dtype], t.numel, self.seed, self.spec.group, t.gen_id, lo, hi, pos, stream)
+        # the library works on its own non-blocking streams: finish the writes first
+        torch.cuda.current_stream().synchronize() if not stream else torch.cuda.ExternalStream(stream).synchronize()
 
     def table(self) -> List[Tuple[str, int, int, int]]:
         return [(t.name, p, t.nbytes, DTYPE_CODE[t.dtype]) for t, p in zip(self.spec.tensors, self.ptrs)]
@@ -57,3 +59,4 @@ class GroupState:
     def scramble(self):
         """Overwrite every tensor (a replacement rank's uninitialised memory)."""
         self.arena.fill_(0xA5)
+        torch.cuda.current_stream().synchronize()
