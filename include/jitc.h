@@ -258,7 +258,8 @@ jitc_status jitc_shard_range(uint64_t n_c, uint32_t k, uint32_t s, uint64_t* c0,
  * comm_job_ranks[i], given the staging geometry.  Output: a 24-B header
  * ('JITP', n_ops, round_bytes, slots) followed by n_ops 48-B operations
  * {round, kind (1 H2D, 2 ALLGATHER, 3 PACK, 4 SEND, 5 RECV, 6 UNPACK,
- * 7 BCAST_DIGESTS), slot, peer, image range [a, b), staging offset, bytes}
+ * 7 DIGEST_SEND, 8 DIGEST_RECV), slot, peer, image range [a, b), staging
+ * offset, bytes}.  Only the group's members get operations
  * (DESIGN.md §8).  Pure: lets the multi-rank schedule be checked without
  * GPUs.  cap == 0 => only *len. */
 jitc_status jitc_restore_plan(const void* selection, size_t sel_len, uint32_t group, int32_t mode,

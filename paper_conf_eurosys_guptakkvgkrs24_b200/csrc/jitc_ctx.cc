@@ -988,13 +988,13 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
   size_t i = 0;
   uint32_t rounds = 0;
   while (i < ops.size()) {
-    if (ops[i].kind == kOpBcastDigests) {
+    if (ops[i].kind == kOpDigestSend || ops[i].kind == kOpDigestRecv) {
       ++i;
       continue;
     }
     const uint32_t j = ops[i].round;
     size_t e = i;
-    while (e < ops.size() && ops[e].round == j && ops[e].kind != kOpBcastDigests) ++e;
+    while (e < ops.size() && ops[e].round == j && ops[e].kind != kOpDigestSend && ops[e].kind != kOpDigestRecv) ++e;
     const uint32_t sl = ops[i].slot;
     ++rounds;
     // 1. host -> device on the copy stream
@@ -1101,6 +1101,15 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
     in.me = c->comm ? c->comm_rank : 0;
     in.staging_bytes = c->staging_bytes;
     in.slot_bytes = c->slot_bytes;
+    if (c->comm) {
+      for (int32_t m : g.members) {
+        int r = comm_rank_of(c, m);
+        if (r >= 0) in.participants.push_back(r);
+      }
+      std::sort(in.participants.begin(), in.participants.end());
+    } else {
+      in.participants = {0};
+    }
     std::vector<PlanOp> ops;
     uint32_t S = 0;
     st = make_plan(c, in, &ops, &S);
@@ -1151,19 +1160,32 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   uint32_t S = 0;
   jitc_status st = make_plan(c, in, &ops, &S);
   if (st) return st;
-  // 1. the lowest writer broadcasts the expected digests (collective over the comm)
-  uint64_t* d_expect = g.d_dig;
-  if (is_writer && my_s == 0) {
-    if (!g.has_fp || g.fp_root != gs.root) return fail(JITC_ESTATE, "jitc_restore: writer fingerprint differs");
-    CU(cudaMemcpyAsync(d_expect, g.fp.data(), g.n_c * 8, cudaMemcpyHostToDevice, c->s_comp));
-  }
-  if (g.n_c) NC(ncclBroadcast(d_expect, d_expect, g.n_c, ncclUint64, in.writers[0], c->comm, c->s_comp));
-  std::vector<uint64_t> want(g.n_c);
-  if (g.n_c) CU(cudaMemcpyAsync(want.data(), d_expect, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
-  CU(cudaStreamSynchronize(c->s_comp));
-  if (root_of(g.layout_hash, want.data(), g.n_c) != gs.root)
-    return fail(JITC_ECORRUPT, "jitc_restore: broadcast digests do not chain to the selected root");
   if (!is_writer && !is_dst) return JITC_OK;
+  // 1. the lowest writer sends the selected class's digests to every destination
+  uint64_t* d_expect = g.d_dig;
+  if (is_writer && (!g.has_fp || g.fp_root != gs.root))
+    return fail(JITC_ESTATE, "jitc_restore: writer fingerprint differs from the selected class");
+  if (is_writer && my_s == 0 && g.n_c)
+    CU(cudaMemcpyAsync(d_expect, g.fp.data(), g.n_c * 8, cudaMemcpyHostToDevice, c->s_comp));
+  bool any = false;
+  for (const PlanOp& op : ops) any |= op.kind == kOpDigestSend || op.kind == kOpDigestRecv;
+  if (any && g.n_c) {
+    NC(ncclGroupStart());
+    for (const PlanOp& op : ops) {
+      if (op.kind == kOpDigestSend) NC(ncclSend(d_expect, g.n_c, ncclUint64, op.peer, c->comm, c->s_comp));
+      if (op.kind == kOpDigestRecv) NC(ncclRecv(d_expect, g.n_c, ncclUint64, op.peer, c->comm, c->s_comp));
+    }
+    NC(ncclGroupEnd());
+  }
+  std::vector<uint64_t> want(g.n_c);
+  if (is_dst) {
+    if (g.n_c) CU(cudaMemcpyAsync(want.data(), d_expect, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
+    CU(cudaStreamSynchronize(c->s_comp));
+    if (root_of(g.layout_hash, want.data(), g.n_c) != gs.root)
+      return fail(JITC_ECORRUPT, "jitc_restore: received digests do not chain to the selected root");
+  } else {
+    want = g.fp;
+  }
   if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
   // 2. data rounds
   st = execute_plan(c, g, ops, S, stats);

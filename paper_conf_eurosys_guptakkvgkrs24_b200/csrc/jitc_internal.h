@@ -226,7 +226,7 @@ uint64_t root_of(uint64_t layout_hash, const uint64_t* d, uint64_t n_c);
 
 // ------------------------------------------------------------------ restore plan (jitc_plan.cc)
 enum : uint8_t { kOpH2D = 1, kOpAllGather = 2, kOpPack = 3, kOpSend = 4, kOpRecv = 5, kOpUnpack = 6,
-                 kOpBcastDigests = 7 };
+                 kOpDigestSend = 7, kOpDigestRecv = 8 };
 constexpr uint32_t kMagicPlan = 0x5054494Au;      // "JITP"
 #pragma pack(push, 1)
 struct PlanOp {      // 48 B
@@ -234,8 +234,8 @@ struct PlanOp {      // 48 B
   uint8_t kind;
   uint8_t slot;      // staging slot (double/multi-buffer index)
   uint16_t pad;
-  int32_t peer;      // comm rank: H2D/PACK = self, SEND/RECV = the other side, UNPACK = block owner,
-                     // BCAST = root
+  int32_t peer;      // comm rank: H2D/PACK = self, SEND/RECV/DIGEST_* = the other side,
+                     // UNPACK = block owner
   uint32_t pad2;
   uint64_t a, b;     // image byte range
   uint64_t off;      // staging byte offset (ALLGATHER: base of the n blocks)
@@ -256,6 +256,7 @@ struct PlanInput {
   uint64_t n_c = 0, chunk_bytes = 0, image_bytes = 0;
   int n = 1, me = 0;                   // communicator size and this rank
   std::vector<int32_t> writers, dests;  // comm ranks (PEER)
+  std::vector<int32_t> participants;    // comm ranks of the group's members, sorted (HOST)
   uint64_t staging_bytes = 0, slot_bytes = 0;
 };
 bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,

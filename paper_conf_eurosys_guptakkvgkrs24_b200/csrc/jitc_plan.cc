@@ -2,13 +2,19 @@
 // this list of operations; jitc_restore_plan exports it so the multi-rank
 // logic can be checked without GPUs (tests/test_multirank_gloo.py).
 //
-// HOST (every rank restarts; reading R17): comm rank r loads
-// chunk range O5(n_c, n, r) of the committed image H2D; every round the ranks
-// all-gather R-byte blocks over NVLink (in place: rank q's block sits at
-// q*R); K3 unpacks every rank's block.
-// PEER (only the replacement lost its state): writer s packs
-// its O5(n_c, k, s) range from live HBM (K2) and sends it to every member
-// that is not a writer; receivers unpack all k blocks (K3).
+// HOST (every rank restarts; reading R17): the n members of
+// the group present in the communicator split the committed image by O5;
+// member q loads chunk range O5(n_c, n, q) H2D; every round the members
+// exchange R-byte blocks over NVLink -- one in-place NCCL all-gather when
+// the group spans the whole communicator, else point-to-point sends/receives
+// among the members only -- and K3 unpacks every member's block.
+// PEER (only the replacement lost its state): the lowest writer
+// sends the digests to every destination; writer s packs its O5(n_c, k, s)
+// range from live HBM (K2) and sends it to every member that is not a
+// writer; receivers unpack all k blocks (K3).
+// Only a group's members take part in its transfers, and every rank handles
+// its groups in increasing group id, so per-group point-to-point traffic
+// cannot form a cycle between ranks (a canonical order, as with locks).
 #include <string.h>
 
 #include <algorithm>
@@ -26,13 +32,22 @@ static void o5_bytes(uint64_t n_c, uint64_t k, uint64_t s, uint64_t C, uint64_t 
 bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
                         std::string* why) {
   ops->clear();
+  *round_bytes = 0;
+  *slots = 0;
   const uint64_t C = in.chunk_bytes, L = in.image_bytes, n_c = in.n_c;
   if (C == 0 || in.n <= 0 || in.me < 0 || in.me >= in.n) {
     *why = "bad plan input";
     return false;
   }
   if (in.mode == JITC_RESTORE_HOST) {
-    const uint64_t n = (uint64_t)in.n;
+    // participants: the group's members present in the communicator (every
+    // rank restarts and holds its own tensors of the group)
+    const std::vector<int32_t>& P = in.participants;
+    const uint64_t n = P.size();
+    const auto it = std::find(P.begin(), P.end(), in.me);
+    if (n == 0 || it == P.end()) return true;  // not a member: nothing to do
+    const uint64_t me = (uint64_t)(it - P.begin());
+    const bool whole_comm = n == (uint64_t)in.n;  // NCCL all-gather over the whole comm, else p2p
     uint64_t R = std::min<uint64_t>(in.slot_bytes, in.staging_bytes / (2 * n)) / C * C;
     if (R == 0) {
       *why = "staging too small for the restore rounds (need >= 2 * n * C bytes)";
@@ -51,12 +66,22 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
     for (uint64_t j = 0; j < J; ++j) {
       const uint32_t sl = (uint32_t)(j % S);
       const uint64_t base = sl * n * R;
-      uint64_t a = q0[in.me] + j * R, b = std::min(q1[in.me], a + R);
-      if (b > a) ops->push_back(PlanOp{(uint32_t)j, kOpH2D, (uint8_t)sl, 0, in.me, 0, a, b, base + in.me * R, b - a});
-      if (n > 1) ops->push_back(PlanOp{(uint32_t)j, kOpAllGather, (uint8_t)sl, 0, -1, 0, 0, 0, base, R});
+      const uint32_t rj = (uint32_t)j;
+      uint64_t a = q0[me] + j * R, b = std::min(q1[me], a + R);
+      if (b > a) ops->push_back(PlanOp{rj, kOpH2D, (uint8_t)sl, 0, in.me, 0, a, b, base + me * R, b - a});
+      if (n > 1 && whole_comm) {
+        ops->push_back(PlanOp{rj, kOpAllGather, (uint8_t)sl, 0, -1, 0, 0, 0, base, R});
+      } else if (n > 1) {
+        for (uint64_t q = 0; q < n; ++q) {
+          if (q == me) continue;
+          if (b > a) ops->push_back(PlanOp{rj, kOpSend, (uint8_t)sl, 0, P[q], 0, a, b, base + me * R, b - a});
+          uint64_t qa = q0[q] + j * R, qb = std::min(q1[q], qa + R);
+          if (qb > qa) ops->push_back(PlanOp{rj, kOpRecv, (uint8_t)sl, 0, P[q], 0, qa, qb, base + q * R, qb - qa});
+        }
+      }
       for (uint64_t q = 0; q < n; ++q) {
         uint64_t qa = q0[q] + j * R, qb = std::min(q1[q], qa + R);
-        if (qb > qa) ops->push_back(PlanOp{(uint32_t)j, kOpUnpack, (uint8_t)sl, 0, (int32_t)q, 0, qa, qb, base + q * R, qb - qa});
+        if (qb > qa) ops->push_back(PlanOp{rj, kOpUnpack, (uint8_t)sl, 0, P[q], 0, qa, qb, base + q * R, qb - qa});
       }
     }
     return true;
@@ -66,11 +91,7 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
     return false;
   }
   const uint64_t k = in.writers.size();
-  if (k == 0) {
-    *round_bytes = 0;
-    *slots = 0;
-    return true;  // dropped group: nothing moves
-  }
+  if (k == 0) return true;  // dropped group: nothing moves
   for (int32_t w : in.writers)
     if (w < 0 || w >= in.n) {
       *why = "a writer is not in the communicator";
@@ -88,8 +109,11 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
   for (uint64_t s = 0; s < k; ++s)
     if (in.writers[s] == in.me) my_s = (int)s;
   const bool is_dst = std::find(in.dests.begin(), in.dests.end(), in.me) != in.dests.end();
-  ops->push_back(PlanOp{0, kOpBcastDigests, 0, 0, in.writers[0], 0, 0, 0, 0, n_c * 8});
   if (in.dests.empty() || (my_s < 0 && !is_dst)) return true;
+  // the lowest writer sends the selected class's digests to every destination
+  if (my_s == 0)
+    for (int32_t d : in.dests) ops->push_back(PlanOp{0, kOpDigestSend, 0, 0, d, 0, 0, 0, 0, n_c * 8});
+  if (is_dst) ops->push_back(PlanOp{0, kOpDigestRecv, 0, 0, in.writers[0], 0, 0, 0, 0, n_c * 8});
   std::vector<uint64_t> q0(k), q1(k);
   uint64_t maxlen = 0;
   for (uint64_t s = 0; s < k; ++s) {
@@ -157,6 +181,11 @@ extern "C" jitc_status jitc_restore_plan(const void* selection, size_t sel_len, 
   in.staging_bytes = staging_bytes;
   in.slot_bytes = slot_bytes;
   for (int32_t w : gs->writers) in.writers.push_back(comm_of(w));
+  for (int32_t m : gs->members) {
+    int r = comm_of(m);
+    if (r >= 0) in.participants.push_back(r);
+  }
+  std::sort(in.participants.begin(), in.participants.end());
   for (int32_t m : gs->members) {
     if (std::find(gs->writers.begin(), gs->writers.end(), m) != gs->writers.end()) continue;
     int r = comm_of(m);

@@ -194,7 +194,8 @@ def parse_selection(sel: bytes) -> dict:
     return out
 
 
-OP_NAMES = {1: "H2D", 2: "ALLGATHER", 3: "PACK", 4: "SEND", 5: "RECV", 6: "UNPACK", 7: "BCAST_DIGESTS"}
+OP_NAMES = {1: "H2D", 2: "ALLGATHER", 3: "PACK", 4: "SEND", 5: "RECV", 6: "UNPACK", 7: "DIGEST_SEND",
+            8: "DIGEST_RECV"}
 
 
 def restore_plan(selection: bytes, group: int, mode: int, comm_job_ranks: Sequence[int], comm_rank: int,
