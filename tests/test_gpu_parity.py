@@ -311,3 +311,53 @@ def test_full_size_sampled(J, shm, cfg):
     ctx.close()
     del states
     torch.cuda.empty_cache()
+
+
+# ------------------------------------------------------------------ edge cases
+def test_edge_empty_tensors_empty_group_max_chunk(J, shm):
+    """Zero-byte tensors inside a table, a group with no tensors at all (L = 0,
+    n_c = 0), 1-byte tensors, and the maximum chunk size (64 MiB) -- capture,
+    restore and verify must all work and stay bit-exact."""
+    g = W.random_table(21, 30, max_bytes=3000, group=1)
+    for i in (0, 7, 29):                           # zero-byte tensors, incl. first and last
+        g.tensors[i].numel = 0
+    g.tensors[3].dtype, g.tensors[3].numel = "u8", 1
+    empty = W.GroupSpec(2, J.REQUIRED, [0], [])
+    for C in (4096, 64 << 20):
+        d = f"{shm}-{C}"
+        st = _state(g, 4)
+        ste = _state(empty, 4)
+        ctx = _ctx(J, C, image_dir=d, staging=2 * C * 2, slot=C)
+        lh, L = ctx.register(1, J.REQUIRED, [0], st.table(), keepalive=st)
+        lh0, L0 = ctx.register(2, J.REQUIRED, [0], ste.table(), keepalive=ste)
+        lay = O.layout_of_group(g, C)
+        assert (lh, L) == (lay.layout_hash, lay.L) and L0 == 0
+        assert lh0 == O.layout_of_group(empty, C).layout_hash
+        blob, sel, cap = _pipeline(J, ctx)
+        recs = _records(blob)
+        assert recs[2].n_c == 0 and recs[2].root == O.root(lh0, np.zeros(0, dtype=np.uint64))
+        assert np.array_equal(recs[1].d, O.jf64(O.pack(O.gen_group(g, 4), lay), C, 0, lay.n_c))
+        st.scramble()
+        ctx.restore(J.ALL_GROUPS, J.HOST)
+        ctx.verify(1)
+        ctx.verify(2)
+        torch.cuda.synchronize()
+        for i, t in enumerate(g.tensors):
+            assert np.array_equal(st.tensor_bytes(i).cpu().numpy(), O.gen_tensor_bytes(t, 4, 1)), t.name
+        ctx.close()
+        shutil.rmtree(d, ignore_errors=True)
+
+
+def test_layout_mismatch_between_replicas(J):
+    """S10 with real fingerprints: one replica registered one tensor with a
+    different size -> ELAYOUT for the whole selection."""
+    import copy
+    g = W.random_table(8, 12)
+    g2 = copy.deepcopy(g)
+    g2.tensors[5].numel += 1
+    a, b = _state(g, 1), _state(g2, 1)
+    ca, cb = _ctx(J, 4096, rank=0, world=2), _ctx(J, 4096, rank=1, world=2)
+    ca.register(0, J.REQUIRED, [0, 1], a.table(), keepalive=a)
+    cb.register(0, J.REQUIRED, [0, 1], b.table(), keepalive=b)
+    st, sel = J.select_consistent_replica(ca.fingerprint() + cb.fingerprint(), [0, 1])
+    assert st == J.ELAYOUT
