@@ -228,6 +228,15 @@ jitc_status jitc_capture(jitc_ctx* ctx, const void* selection, size_t sel_len, u
  * the lowest-rank writer of each group writes it. */
 jitc_status jitc_commit(jitc_ctx* ctx, const void* selection, size_t sel_len);
 
+/* Local (non-collective) capture of every held group by this rank alone:
+ * fingerprint -> select over its own record -> capture (k = 1) -> commit.
+ * The paper's user-level protocol in which each healthy rank saves its own
+ * state, and the host round trip of transient
+ * recovery (copy to host, reset, copy back).  A DIRTY group
+ * makes it fail with JITC_ENOCONSISTENT.  This is what the
+ * watchdog runs with JITC_ON_HANG_LOCAL_CAPTURE. */
+jitc_status jitc_capture_local(jitc_ctx* ctx, jitc_stats* stats);
+
 /* ---- restore ------------------------------------------------------------- */
 /* A9-A11.  HOST: refuses an uncommitted image (JITC_EINCOMPLETE); each comm
  * rank loads chunk range O5(n_c, n, r) H2D, the ranks all-gather the slices

@@ -1369,6 +1369,15 @@ static void stop_thread(jitc_ctx* c) {
   if (c->wthread.joinable()) c->wthread.join();
 }
 
+jitc_status jitc_capture_local(jitc_ctx* c, jitc_stats* stats) {
+  if (!c) return fail(JITC_EINVAL, "jitc_capture_local: null ctx");
+  jitc_stats st{};
+  st.first_bad_chunk = -1;
+  jitc_status r = local_capture(c, &st);
+  if (stats) *stats = st;
+  return r;
+}
+
 jitc_status jitc_watch_event(jitc_ctx* c, void* event, uint64_t tag) {
   if (!c || !event) return fail(JITC_EINVAL, "jitc_watch_event: null argument");
   std::lock_guard<std::mutex> lk(c->wmu);

@@ -109,6 +109,7 @@ def lib() -> ctypes.CDLL:
         "jitc_inject_hang": ([vp, i32, u32], i32),
         "jitc_inject_release": ([u32], i32),
         "jitc_watch_event": ([vp, vp, u64], i32),
+        "jitc_capture_local": ([vp, P(Stats)], i32),
         "jitc_watchdog_start": ([vp, u32, i32, vp, vp], i32),
         "jitc_watchdog_wait": ([vp, u32, P(i32), P(u64), P(ctypes.c_double), P(ctypes.c_double), P(Stats)], i32),
         "jitc_watchdog_stop": ([vp], i32),
@@ -127,7 +128,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
-            "jitc_inject_release", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
+            "jitc_inject_release", "jitc_capture_local", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE = 0, 1
 
@@ -337,6 +338,11 @@ class Context:
     def capture(self, selection: bytes, group: int = ALL_GROUPS) -> dict:
         st = Stats()
         _check(self._L.jitc_capture(self._h, selection, len(selection), group, ctypes.byref(st)), "jitc_capture")
+        return st.as_dict()
+
+    def capture_local(self) -> dict:
+        st = Stats()
+        _check(self._L.jitc_capture_local(self._h, ctypes.byref(st)), "jitc_capture_local")
         return st.as_dict()
 
     def commit(self, selection: bytes):
