@@ -299,6 +299,19 @@ jitc_status jitc_watchdog_wait(jitc_ctx* ctx, uint32_t max_ms, int32_t* fired, u
                                double* action_ms, jitc_stats* action_stats);
 jitc_status jitc_watchdog_stop(jitc_ctx* ctx);
 
+/* ---- analytic model (NEXT-3; §5, eqs. 1-8) ------------------------ */
+enum { JITC_MODEL_PERIODIC_OPTIMAL = 0, JITC_MODEL_PERIODIC = 1, JITC_MODEL_USER_JIT = 2,
+       JITC_MODEL_TRANSPARENT_JIT = 3 };
+/* Wasted GPU time per GPU per unit of useful time (w) and the wasted-time
+ * fraction w_f = w / (1 + w) (eq. 6) for N GPUs with per-GPU failure rate f
+ * (1/s), checkpoint time o (s), fixed recovery time r (s), minibatch time m
+ * (s), JIT steady-state overhead o_jit (fraction) and, for
+ * JITC_MODEL_PERIODIC, checkpoint frequency c (1/s).  *c_opt (may be NULL)
+ * receives the optimal periodic frequency c* = sqrt(N f / (2 o)) (eq. 3; the
+ * printed "2α" is read as 2o).  Pure. */
+jitc_status jitc_waste_model(int32_t kind, double n_gpus, double f, double o, double r, double m, double o_jit,
+                             double c, double* c_opt, double* w, double* w_f);
+
 /* ---- counters ---------------------------------------------------------------- */
 jitc_status jitc_kernel_counters(jitc_ctx* ctx, int32_t kind, jitc_kernel_counter* out);
 jitc_status jitc_reset_counters(jitc_ctx* ctx);

@@ -110,6 +110,7 @@ def lib() -> ctypes.CDLL:
         "jitc_inject_release": ([u32], i32),
         "jitc_watch_event": ([vp, vp, u64], i32),
         "jitc_capture_local": ([vp, P(Stats)], i32),
+        "jitc_waste_model": ([i32] + [ctypes.c_double] * 7 + [P(ctypes.c_double)] * 3, i32),
         "jitc_watchdog_start": ([vp, u32, i32, vp, vp], i32),
         "jitc_watchdog_wait": ([vp, u32, P(i32), P(u64), P(ctypes.c_double), P(ctypes.c_double), P(Stats)], i32),
         "jitc_watchdog_stop": ([vp], i32),
@@ -128,7 +129,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
-            "jitc_inject_release", "jitc_capture_local", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
+            "jitc_inject_release", "jitc_capture_local", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE = 0, 1
 
@@ -193,6 +194,18 @@ def parse_selection(sel: bytes) -> dict:
                                   excluded=[(ints[k + n_mem + 2 * j], ints[k + n_mem + 2 * j + 1]) for j in range(n_ex)],
                                   conflict_chunks=cf, layout_hash=lh, chunk_bytes=C, n_c=n_c, image_bytes=L, root=root))
     return out
+
+
+MODEL_PERIODIC_OPTIMAL, MODEL_PERIODIC, MODEL_USER_JIT, MODEL_TRANSPARENT_JIT = 0, 1, 2, 3
+
+
+def waste_model(kind: int, n_gpus: float, f: float, o: float = 0.0, r: float = 0.0, m: float = 0.0,
+                o_jit: float = 0.0, c: float = 0.0) -> dict:
+    """PAPER.md §5 eqs. 1-8 through the C ABI: {c_opt, w, w_f}."""
+    co, w, wf = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+    _check(lib().jitc_waste_model(kind, n_gpus, f, o, r, m, o_jit, c, ctypes.byref(co), ctypes.byref(w),
+                                  ctypes.byref(wf)), "jitc_waste_model")
+    return dict(c_opt=co.value, w=w.value, w_f=wf.value)
 
 
 OP_NAMES = {1: "H2D", 2: "ALLGATHER", 3: "PACK", 4: "SEND", 5: "RECV", 6: "UNPACK", 7: "DIGEST_SEND",
