@@ -140,7 +140,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    from oracle import oracle as O
+    from workloads import configs as W
     g2, lay, ts, total = oracle_sample(args.config, args.ref_sample << 20)
     for _ in range(args.warmup):
         oracle_step(lay, ts)
@@ -153,7 +153,8 @@ def run_reference(args):
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic (O9 counter-based generator)",
-            "config": {"workload": f"{args.config} (bounded sample)", "sample_bytes": lay.L},
+            "config": {"workload": W.CONFIGS[args.config]().name, "sample_bytes": lay.L,
+                       "note": "bounded prefix of the same workload's REQUIRED image; oracle pack+JF64+JF64+unpack"},
             "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
                              "sample": f"first {lay.L / 2**20:.0f} MiB of the {args.config} REQUIRED-group image"},
             "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}

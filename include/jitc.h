@@ -276,6 +276,19 @@ jitc_status jitc_restore_plan(const void* selection, size_t sel_len, uint32_t gr
                               uint64_t staging_bytes, uint64_t slot_bytes, void* plan, size_t cap,
                               size_t* len);
 
+/* ---- durable tier (NEXT-4; §6.3) ---------------------- */
+/* Streams the committed host image of `group` to `dir` (parallel O_DIRECT
+ * writes when the file system supports them, then fdatasync), then the
+ * manifest, then LAST the commit record -- the low-frequency periodic copy
+ * that survives losing every replica, in the same format.
+ * JITC_EINCOMPLETE if the group has no committed checkpoint. */
+jitc_status jitc_persist(jitc_ctx* ctx, uint32_t group, const char* dir, jitc_stats* stats);
+/* Reads a durable copy back into the host image (validating the commit
+ * record, the manifest trailer and the layout: JITC_EINCOMPLETE /
+ * JITC_ELAYOUT) and installs its manifest, so that jitc_restore(HOST)
+ * restores it with full K3 verification. */
+jitc_status jitc_stage_in(jitc_ctx* ctx, uint32_t group, const char* dir, jitc_stats* stats);
+
 /* ---- hang detection (NEXT-1; §3.1-3.2) ------------------ */
 /* The caller records a CUDA event after each collective on its NCCL stream
  * (the event the compute stream waits on, PAPER.md:122 / Fig. 3) and puts it

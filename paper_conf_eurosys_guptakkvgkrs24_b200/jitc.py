@@ -110,6 +110,8 @@ def lib() -> ctypes.CDLL:
         "jitc_inject_release": ([u32], i32),
         "jitc_watch_event": ([vp, vp, u64], i32),
         "jitc_capture_local": ([vp, P(Stats)], i32),
+        "jitc_persist": ([vp, u32, ctypes.c_char_p, P(Stats)], i32),
+        "jitc_stage_in": ([vp, u32, ctypes.c_char_p, P(Stats)], i32),
         "jitc_waste_model": ([i32] + [ctypes.c_double] * 7 + [P(ctypes.c_double)] * 3, i32),
         "jitc_watchdog_start": ([vp, u32, i32, vp, vp], i32),
         "jitc_watchdog_wait": ([vp, u32, P(i32), P(u64), P(ctypes.c_double), P(ctypes.c_double), P(Stats)], i32),
@@ -129,7 +131,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
-            "jitc_inject_release", "jitc_capture_local", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
+            "jitc_inject_release", "jitc_capture_local", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE = 0, 1
 
@@ -356,6 +358,16 @@ class Context:
     def capture_local(self) -> dict:
         st = Stats()
         _check(self._L.jitc_capture_local(self._h, ctypes.byref(st)), "jitc_capture_local")
+        return st.as_dict()
+
+    def persist(self, group: int, directory: str) -> dict:
+        st = Stats()
+        _check(self._L.jitc_persist(self._h, group, directory.encode(), ctypes.byref(st)), "jitc_persist")
+        return st.as_dict()
+
+    def stage_in(self, group: int, directory: str) -> dict:
+        st = Stats()
+        _check(self._L.jitc_stage_in(self._h, group, directory.encode(), ctypes.byref(st)), "jitc_stage_in")
         return st.as_dict()
 
     def commit(self, selection: bytes):
