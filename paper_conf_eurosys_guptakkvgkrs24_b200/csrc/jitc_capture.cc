@@ -1,0 +1,212 @@
+// libjitc.so capture path: A7 capture (K2 gather-pack + D2H, shard s of k),
+// A8 commit (manifest, then the commit record LAST -- PAPER.md:136), and the
+// local non-collective capture used by transient recovery and the watchdog
+// (PAPER.md:105-108, :173).
+#include "jitc_ctx.h"
+
+using namespace jitc;
+
+// ------------------------------------------------------------ capture (K2 + D2H)
+static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelection& gs, uint64_t v_star,
+                                 jitc_stats* stats) {
+  auto it = std::find(gs.writers.begin(), gs.writers.end(), c->cfg.rank);
+  if (it == gs.writers.end()) return JITC_OK;  // not a writer
+  uint64_t s = (uint64_t)(it - gs.writers.begin()), k = gs.writers.size();
+  if (!g.has_fp) return fail(JITC_ESTATE, "jitc_capture: group " + std::to_string(g.id) + " not fingerprinted");
+  if (gs.layout_hash != g.layout_hash || gs.n_c != g.n_c || gs.image_bytes != g.L)
+    return fail(JITC_ELAYOUT, "jitc_capture: selection layout differs from the registered one");
+  if (g.fp_version != v_star || g.fp_root != gs.root || g.fp_phase != JITC_PHASE_CLEAN)
+    return fail(JITC_ESTATE, "jitc_capture: this rank's fingerprint is not the selected candidate");
+  uint64_t c0, c1;
+  shard_range(g.n_c, k, s, &c0, &c1);
+  uint64_t b0 = std::min(c0 * g.C, g.L), b1 = std::min(c1 * g.C, g.L);
+  // the lowest writer invalidates the previous commit before any byte changes
+  if (s == 0 && g.img_shm) unlink(gpath(c, g.id, ".commit").c_str());
+  g.commit_priv.clear();
+  if (b1 > b0) {
+    CU(cudaMemsetAsync(g.d_dig2 + c0, 0, (c1 - c0) * 8, c->s_comp));
+    const bool zc = (c->cfg.flags & JITC_F_ZERO_COPY_D2H) != 0;
+    if (zc) {
+      uint32_t lo, hi;
+      seg_span(g, b0, b1, &lo, &hi);
+      jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, g.img_d, 0), g.d_dig2, b1 - b0);
+      if (st) return st;
+      if (stats) stats->rounds += 1;
+    } else {
+      const uint64_t R = c->slot_bytes;
+      const int nslots = (int)std::min<uint64_t>(jitc_ctx::kSlots, c->staging_bytes / R);
+      uint32_t j = 0;
+      for (uint64_t a = b0; a < b1; a += R, ++j) {
+        uint64_t b = std::min(a + R, b1);
+        int sl = (int)(j % nslots);
+        uint8_t* slot = c->staging + sl * R;
+        if (j >= (uint32_t)nslots) CU(cudaStreamWaitEvent(c->s_comp, c->ev_free[sl], 0));
+        uint32_t lo, hi;
+        seg_span(g, a, b, &lo, &hi);
+        jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, slot, a), g.d_dig2, b - a);
+        if (st) return st;
+        CU(cudaEventRecord(c->ev_ready[sl], c->s_comp));
+        CU(cudaStreamWaitEvent(c->s_copy, c->ev_ready[sl], 0));
+        CU(cudaMemcpyAsync(g.img_h + a, slot, b - a, cudaMemcpyDeviceToHost, c->s_copy));
+        CU(cudaEventRecord(c->ev_free[sl], c->s_copy));
+      }
+      if (stats) stats->rounds += j;
+      CU(cudaEventRecord(c->ev_join, c->s_copy));
+      CU(cudaStreamWaitEvent(c->s_comp, c->ev_join, 0));
+      if (stats) stats->d2h_bytes += b1 - b0;
+    }
+    CU(cudaMemcpyAsync(c->h_dig, g.d_dig2 + c0, (c1 - c0) * 8, cudaMemcpyDeviceToHost, c->s_comp));
+  }
+  CU(cudaStreamSynchronize(c->s_comp));
+  for (uint64_t ch = c0; ch < c1; ++ch)
+    if (c->h_dig[ch - c0] != g.fp[ch])
+      return fail(JITC_EUNSTABLE, "jitc_capture: group " + std::to_string(g.id) + " chunk " + std::to_string(ch) +
+                                      " changed between fingerprint and capture");
+  g.captured = true;
+  g.cap_v = v_star;
+  if (stats) stats->image_bytes += b1 - b0;
+  return JITC_OK;
+}
+
+jitc_status jitc_capture(jitc_ctx* c, const void* selection, size_t sel_len, uint32_t group, jitc_stats* stats) {
+  if (!c) return fail(JITC_EINVAL, "jitc_capture: null ctx");
+  Selection sel;
+  std::string why;
+  if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
+    return fail(JITC_EINVAL, "jitc_capture: " + why);
+  if (sel.status != JITC_OK) return fail(sel.status, "jitc_capture: selection status is not OK");
+  CU(cudaSetDevice(c->device));
+  if (stats) memset(stats, 0, sizeof *stats), stats->first_bad_chunk = -1;
+  CallTimer t(c);
+  CU(cudaEventRecord(c->ev_t0, c->s_comp));
+  for (auto& kv : c->groups) {
+    GroupState& g = kv.second;
+    if (!g.held || (group != JITC_ALL_GROUPS && g.id != group)) continue;
+    const GroupSelection* gs = sel.find(g.id);
+    if (!gs) return fail(JITC_ELAYOUT, "jitc_capture: group missing from selection");
+    jitc_status st = capture_group(c, g, *gs, sel.v_star, stats);
+    if (st) return st;
+  }
+  CU(cudaEventRecord(c->ev_t1, c->s_comp));
+  CU(cudaEventSynchronize(c->ev_t1));
+  finish_stats(c, t, stats, true);
+  return JITC_OK;
+}
+
+// ------------------------------------------------------------ commit (manifest, then commit record)
+static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelection& gs, uint64_t v_star) {
+  std::vector<uint8_t> b;
+  ManifestHdr h{};
+  h.magic = kMagicManifest;
+  h.fmt = 1;
+  h.group = g.id;
+  h.n_tensors = (uint32_t)g.t.size();
+  h.v_star = v_star;
+  h.layout_hash = g.layout_hash;
+  h.chunk_bytes = g.C;
+  h.n_c = g.n_c;
+  h.image_bytes = g.L;
+  h.k = (uint32_t)gs.writers.size();
+  auto put = [&](const void* p, size_t n) { b.insert(b.end(), (const uint8_t*)p, (const uint8_t*)p + n); };
+  auto pad = [&]() { while (b.size() % 8) b.push_back(0); };
+  put(&h, sizeof h);
+  put(gs.writers.data(), 4 * gs.writers.size());
+  pad();
+  for (size_t i = 0; i < g.t.size(); ++i) {
+    uint16_t ln = (uint16_t)g.names[i].size();
+    put(&ln, 2);
+    put(g.names[i].data(), ln);
+    uint32_t dt = g.t[i].dtype;
+    uint64_t nb = g.t[i].nbytes, off = g.off[i];
+    put(&dt, 4);
+    put(&nb, 8);
+    put(&off, 8);
+  }
+  pad();
+  put(g.fp.data(), 8 * g.n_c);
+  put(&g.fp_root, 8);
+  for (size_t s = 0; s < gs.writers.size(); ++s) {
+    ShardEnt e{};
+    e.writer = gs.writers[s];
+    shard_range(g.n_c, gs.writers.size(), s, &e.c0, &e.c1);
+    put(&e, sizeof e);
+  }
+  uint64_t tr = manifest_trailer(b.data(), b.size());
+  put(&tr, 8);
+  return b;
+}
+
+jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len, bool collective) {
+  if (!c) return fail(JITC_EINVAL, "jitc_commit: null ctx");
+  Selection sel;
+  std::string why;
+  if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
+    return fail(JITC_EINVAL, "jitc_commit: " + why);
+  if (sel.status != JITC_OK) return fail(sel.status, "jitc_commit: selection status is not OK");
+  CU(cudaSetDevice(c->device));
+  jitc_status st = collective ? barrier(c) : JITC_OK;  // every writer's capture has returned
+  if (st) return st;
+  for (auto& kv : c->groups) {
+    GroupState& g = kv.second;
+    if (!g.held) continue;
+    const GroupSelection* gs = sel.find(g.id);
+    if (!gs || gs->writers.empty()) continue;
+    bool writer = std::find(gs->writers.begin(), gs->writers.end(), c->cfg.rank) != gs->writers.end();
+    if (!writer) continue;
+    if (!g.captured || g.cap_v != sel.v_star) return fail(JITC_ESTATE, "jitc_commit: group not captured at v*");
+    std::vector<uint8_t> man = build_manifest(g, *gs, sel.v_star);
+    CommitRec cr{};
+    cr.magic = kMagicCommit;
+    cr.group = g.id;
+    cr.v_star = sel.v_star;
+    memcpy(&cr.trailer, man.data() + man.size() - 8, 8);
+    cr.manifest_bytes = man.size();
+    g.man_d = g.fp;
+    g.man_root = g.fp_root;
+    g.has_man = true;
+    g.man_priv = man;
+    g.commit_priv.assign((uint8_t*)&cr, (uint8_t*)&cr + sizeof cr);
+    if (g.img_shm && gs->writers[0] == c->cfg.rank) {
+      if (!write_file_atomic(gpath(c, g.id, ".manifest"), man.data(), man.size()))
+        return fail(JITC_EIO, "jitc_commit: writing manifest: " + std::string(strerror(errno)));
+      if (!write_file_atomic(gpath(c, g.id, ".commit"), (const uint8_t*)&cr, sizeof cr))
+        return fail(JITC_EIO, "jitc_commit: writing commit record: " + std::string(strerror(errno)));
+    }
+  }
+  return collective ? barrier(c) : JITC_OK;  // nobody restores before every commit record exists
+}
+
+jitc_status jitc_commit(jitc_ctx* c, const void* selection, size_t sel_len) {
+  return commit_impl(c, selection, sel_len, true);
+}
+
+jitc_status jitc::local_capture(jitc_ctx* c, jitc_stats* st) {
+  size_t len = 0;
+  jitc_status r = jitc_fingerprint(c, JITC_ALL_GROUPS, nullptr, 0, &len);
+  if (r) return r;
+  std::vector<uint8_t> blob(len);
+  r = jitc_fingerprint(c, JITC_ALL_GROUPS, blob.data(), blob.size(), &len);
+  if (r) return r;
+  int32_t me = c->cfg.rank;
+  size_t sl = 0;
+  jitc_select_consistent_replica(blob.data(), len, &me, 1, nullptr, 0, &sl);
+  std::vector<uint8_t> sel(sl);
+  r = jitc_select_consistent_replica(blob.data(), len, &me, 1, sel.data(), sel.size(), &sl);
+  if (r) return r;
+  r = jitc_capture(c, sel.data(), sl, JITC_ALL_GROUPS, st);
+  if (r) return r;
+  return commit_impl(c, sel.data(), sl, false);
+}
+
+extern "C" {
+
+jitc_status jitc_capture_local(jitc_ctx* c, jitc_stats* stats) {
+  if (!c) return fail(JITC_EINVAL, "jitc_capture_local: null ctx");
+  jitc_stats st{};
+  st.first_bad_chunk = -1;
+  jitc_status r = local_capture(c, &st);
+  if (stats) *stats = st;
+  return r;
+}
+
+}  // extern "C"

@@ -1,0 +1,317 @@
+// Internal definitions shared by the libjitc.so context sources
+// (jitc_ctx.cc, jitc_capture.cc, jitc_restore.cc, jitc_durable.cc,
+// jitc_watchdog.cc): the context and group state, and small helpers.
+#pragma once
+
+#include <cuda.h>
+#include <errno.h>
+#include <fcntl.h>
+#include <nccl.h>
+#include <stdio.h>
+#include <string.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <sys/types.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <chrono>
+#include <condition_variable>
+#include <mutex>
+#include <thread>
+#include <map>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "jitc_internal.h"
+
+
+namespace jitc {
+
+struct GroupState {
+  uint32_t id = 0;
+  int policy = JITC_REQUIRED;
+  std::vector<int32_t> members;
+  bool held = false;
+  int slot = -1;  // phase-word slot
+  // layout (held groups)
+  std::vector<std::string> names;
+  std::vector<jitc_tensor> t;
+  std::vector<uint64_t> off;
+  uint64_t C = 0, L = 0, n_c = 0, layout_hash = 0;
+  std::vector<Seg> segs;
+  Seg* d_segs = nullptr;
+  uint64_t* d_dig = nullptr;   // K1 digests
+  uint64_t* d_dig2 = nullptr;  // K2 / K3 digests
+  // last fingerprint
+  bool has_fp = false;
+  std::vector<uint64_t> fp;
+  uint64_t fp_root = 0, fp_version = 0;
+  int fp_phase = 0;
+  // last capture
+  bool captured = false;
+  uint64_t cap_v = 0;
+  // manifest digests (after commit / restore) for jitc_verify
+  bool has_man = false;
+  std::vector<uint64_t> man_d;
+  uint64_t man_root = 0;
+  // host image
+  uint8_t* img_h = nullptr;
+  uint8_t* img_d = nullptr;  // device alias of the mapped host image
+  size_t img_bytes = 0;
+  bool img_shm = false;
+  std::string img_path;
+  std::vector<uint8_t> man_priv, commit_priv;  // private-memory manifest / commit
+};
+
+typedef CUresult (*PFN_writeValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+
+}  // namespace jitc
+
+using namespace jitc;
+
+struct jitc_ctx {
+  jitc_config cfg{};
+  std::string image_dir;
+  int device = 0;
+  cudaStream_t s_comp = nullptr, s_copy = nullptr;
+  bool own_streams = false;
+  uint8_t* staging = nullptr;
+  uint64_t staging_bytes = 0, slot_bytes = 0;
+  bool own_staging = false;
+  static constexpr int kSlots = 8;
+  cudaEvent_t ev_ready[kSlots]{}, ev_free[kSlots]{};
+  cudaEvent_t ev_t0 = nullptr, ev_t1 = nullptr, ev_join = nullptr;
+  std::vector<cudaEvent_t> kev;  // kernel timing pairs
+  std::vector<int> kev_kind;
+  std::vector<uint64_t> kev_bytes;
+  size_t kev_used = 0;
+  uint64_t* phase_h = nullptr;
+  uint64_t* phase_d = nullptr;
+  int phase_used = 0;
+  PFN_writeValue64 write_value64 = nullptr;
+  std::map<uint32_t, GroupState> groups;
+  uint64_t* h_dig = nullptr;  // pinned digest scratch
+  size_t h_dig_n = 0;
+  int grid = 0;
+  // communicator
+  ncclComm_t comm = nullptr;
+  int comm_n = 0, comm_rank = -1;
+  std::vector<int32_t> comm_job;  // comm rank -> job rank
+  uint64_t* d_small = nullptr;    // 64 B device scratch for size exchange / barrier
+  uint32_t* d_work = nullptr;     // K1/K2/K3 batch counters (self-resetting)
+  uint64_t* h_small = nullptr;    // pinned
+  // watchdog (NEXT-1): explicit event watch-list polled by a native thread
+  struct Watch {
+    cudaEvent_t ev;
+    uint64_t tag;
+    double t_added;
+  };
+  std::mutex wmu;
+  std::condition_variable wcv;
+  std::vector<Watch> watches;
+  std::thread wthread;
+  bool wrun = false, fired = false, action_done = false;
+  uint64_t fired_tag = 0;
+  double detect_ms = 0, waited_ms = 0, action_ms = 0;
+  uint32_t timeout_ms = 0;
+  int action = 0;
+  jitc_hang_fn hang_fn = nullptr;
+  void* hang_user = nullptr;
+  jitc_status action_status = JITC_OK;
+  jitc_stats action_stats{};
+  // counters
+  jitc_kernel_counter kc[4]{};
+  uint64_t launches_in_call = 0;
+  double kernel_ms_in_call = 0;
+};
+
+// ----------------------------------------------------------------- helpers
+namespace jitc {
+
+inline jitc_status fail(jitc_status st, const std::string& msg) {
+  set_error(msg);
+  return st;
+}
+
+#define CU(call)                                                                                  \
+  do {                                                                                            \
+    cudaError_t e_ = (call);                                                                      \
+    if (e_ != cudaSuccess)                                                                        \
+      return fail(JITC_ECUDA, std::string(__func__) + ": " #call ": " + cudaGetErrorString(e_)); \
+  } while (0)
+#define NC(call)                                                                                  \
+  do {                                                                                            \
+    ncclResult_t r_ = (call);                                                                     \
+    if (r_ != ncclSuccess)                                                                        \
+      return fail(JITC_ENCCL, std::string(__func__) + ": " #call ": " + ncclGetErrorString(r_));  \
+  } while (0)
+
+inline double now_ms() {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+struct CallTimer {
+  jitc_ctx* c;
+  double t0;
+  explicit CallTimer(jitc_ctx* ctx) : c(ctx), t0(now_ms()) {
+    c->launches_in_call = 0;
+    c->kernel_ms_in_call = 0;
+    c->kev_used = 0;
+  }
+};
+
+// Kernel launch with optional event bracketing (JITC_F_TIME_KERNELS).
+inline jitc_status run_segments(jitc_ctx* c, GroupState& g, int mode, const LaunchRanges& r, uint64_t* dig,
+                         uint64_t bytes) {
+  bool timed = (c->cfg.flags & JITC_F_TIME_KERNELS) && c->kev_used + 2 <= c->kev.size();
+  if (timed) CU(cudaEventRecord(c->kev[c->kev_used], c->s_comp));
+  CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->d_work, c->s_comp));
+  if (timed) {
+    CU(cudaEventRecord(c->kev[c->kev_used + 1], c->s_comp));
+    c->kev_kind[c->kev_used / 2] = mode;
+    c->kev_bytes[c->kev_used / 2] = bytes;
+    c->kev_used += 2;
+  }
+  c->launches_in_call++;
+  c->kc[mode].launches++;
+  c->kc[mode].bytes += bytes;
+  return JITC_OK;
+}
+
+// After the call's work has completed: harvest kernel timings into counters.
+inline void harvest(jitc_ctx* c) {
+  for (size_t i = 0; i + 1 < c->kev_used; i += 2) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, c->kev[i], c->kev[i + 1]) == cudaSuccess) {
+      c->kc[c->kev_kind[i / 2]].ms += ms;
+      c->kernel_ms_in_call += ms;
+    }
+  }
+  c->kev_used = 0;
+}
+
+inline void finish_stats(jitc_ctx* c, const CallTimer& t, jitc_stats* st, bool device_span) {
+  harvest(c);
+  if (!st) return;
+  st->ms_host = now_ms() - t.t0;
+  st->ms_kernel = c->kernel_ms_in_call;
+  st->kernel_launches = c->launches_in_call;
+  if (device_span) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, c->ev_t0, c->ev_t1) == cudaSuccess) st->ms_device = ms;
+  }
+}
+
+// Segments whose image offset lies in [a, b) (segments never straddle a chunk
+// boundary and rounds are chunk-aligned, so this is exact).
+inline void seg_span(const GroupState& g, uint64_t a, uint64_t b, uint32_t* lo, uint32_t* hi) {
+  auto cmp = [](const Seg& s, uint64_t v) { return s.img_off < v; };
+  *lo = (uint32_t)(std::lower_bound(g.segs.begin(), g.segs.end(), a, cmp) - g.segs.begin());
+  *hi = (uint32_t)(std::lower_bound(g.segs.begin(), g.segs.end(), b, cmp) - g.segs.begin());
+}
+
+inline LaunchRanges one_range(uint32_t lo, uint32_t hi, const void* base, uint64_t base_off) {
+  LaunchRanges r{};
+  r.n = 1;
+  r.seg_begin[0] = lo;
+  r.seg_end[0] = hi;
+  r.prefix[0] = 0;
+  r.prefix[1] = hi - lo;
+  r.base[0] = (uint64_t)base;
+  r.base_off[0] = base_off;
+  return r;
+}
+
+inline void add_range(LaunchRanges& r, uint32_t lo, uint32_t hi, const void* base, uint64_t base_off) {
+  r.seg_begin[r.n] = lo;
+  r.seg_end[r.n] = hi;
+  r.base[r.n] = (uint64_t)base;
+  r.base_off[r.n] = base_off;
+  r.prefix[r.n + 1] = r.prefix[r.n] + (hi - lo);
+  r.n++;
+}
+
+inline jitc_status ensure_h_dig(jitc_ctx* c, size_t n) {
+  if (n <= c->h_dig_n) return JITC_OK;
+  if (c->h_dig) cudaFreeHost(c->h_dig);
+  c->h_dig = nullptr;
+  c->h_dig_n = 0;
+  CU(cudaHostAlloc(&c->h_dig, std::max<size_t>(n, 1) * 8, cudaHostAllocDefault));
+  c->h_dig_n = n;
+  return JITC_OK;
+}
+
+inline void free_group(GroupState& g) {
+  if (g.d_segs) cudaFree(g.d_segs);
+  if (g.d_dig) cudaFree(g.d_dig);
+  if (g.d_dig2) cudaFree(g.d_dig2);
+  if (g.img_h) {
+    if (g.img_shm) {
+      cudaHostUnregister(g.img_h);
+      munmap(g.img_h, g.img_bytes);
+    } else {
+      cudaFreeHost(g.img_h);
+    }
+  }
+  g.d_segs = nullptr;
+  g.d_dig = g.d_dig2 = nullptr;
+  g.img_h = g.img_d = nullptr;
+}
+
+inline std::string gpath(const jitc_ctx* c, uint32_t g, const char* ext) {
+  return c->image_dir + "/g" + std::to_string(g) + ext;
+}
+
+inline std::vector<TopoEntry> topology(const jitc_ctx* c) {
+  std::vector<TopoEntry> t;
+  for (auto& kv : c->groups) t.push_back(TopoEntry{kv.first, kv.second.policy, kv.second.members});
+  return t;
+}
+
+inline int comm_rank_of(const jitc_ctx* c, int32_t job) {
+  for (int i = 0; i < c->comm_n; ++i)
+    if (c->comm_job[i] == job) return i;
+  return -1;
+}
+
+inline bool write_file_atomic(const std::string& path, const uint8_t* p, size_t n) {
+  std::string tmp = path + ".tmp";
+  FILE* f = fopen(tmp.c_str(), "wb");
+  if (!f) return false;
+  bool ok = fwrite(p, 1, n, f) == n;
+  ok = (fflush(f) == 0) && ok;
+  ok = (fsync(fileno(f)) == 0) && ok;
+  fclose(f);
+  return ok && rename(tmp.c_str(), path.c_str()) == 0;
+}
+
+inline bool read_file(const std::string& path, std::vector<uint8_t>* out) {
+  FILE* f = fopen(path.c_str(), "rb");
+  if (!f) return false;
+  fseek(f, 0, SEEK_END);
+  long n = ftell(f);
+  fseek(f, 0, SEEK_SET);
+  out->resize(n > 0 ? (size_t)n : 0);
+  bool ok = n <= 0 || fread(out->data(), 1, (size_t)n, f) == (size_t)n;
+  fclose(f);
+  return ok;
+}
+
+inline jitc_status barrier(jitc_ctx* c) {
+  if (!c->comm) return JITC_OK;
+  NC(ncclAllReduce(c->d_small, c->d_small + 1, 1, ncclUint64, ncclSum, c->comm, c->s_comp));
+  CU(cudaStreamSynchronize(c->s_comp));
+  return JITC_OK;
+}
+
+}  // namespace jitc
+
+namespace jitc {
+// defined in jitc_capture.cc
+jitc_status commit_impl(jitc_ctx* c, const void* selection, size_t sel_len, bool collective);
+jitc_status local_capture(jitc_ctx* c, jitc_stats* st);
+// defined in jitc_ctx.cc
+jitc_status fingerprint_group(jitc_ctx* c, GroupState& g);
+}  // namespace jitc

@@ -1,0 +1,381 @@
+// libjitc.so restore path: A9-A11 (HOST: H2D slices + NVLink exchange + K3
+// unpack+verify; PEER: K2 from the writers' live HBM over NVLink + K3) executed
+// from an explicit round plan (jitc_plan.cc), and A12 verify.
+#include "jitc_ctx.h"
+
+using namespace jitc;
+
+// ------------------------------------------------------------ restore
+struct ManifestView {
+  ManifestHdr h;
+  std::vector<int32_t> writers;
+  std::vector<uint64_t> d;
+  uint64_t root = 0;
+};
+
+static jitc_status load_manifest(jitc_ctx* c, GroupState& g, ManifestView* mv) {
+  std::vector<uint8_t> man, com;
+  if (g.img_shm) {
+    if (!read_file(gpath(c, g.id, ".commit"), &com) || !read_file(gpath(c, g.id, ".manifest"), &man))
+      return fail(JITC_EINCOMPLETE, "jitc_restore: group " + std::to_string(g.id) + " has no committed checkpoint");
+  } else {
+    man = g.man_priv;
+    com = g.commit_priv;
+  }
+  if (com.size() != sizeof(CommitRec) || man.size() < sizeof(ManifestHdr) + 16)
+    return fail(JITC_EINCOMPLETE, "jitc_restore: missing or torn manifest / commit record");
+  CommitRec cr;
+  memcpy(&cr, com.data(), sizeof cr);
+  uint64_t tr_stored;
+  memcpy(&tr_stored, man.data() + man.size() - 8, 8);
+  if (cr.magic != kMagicCommit || cr.manifest_bytes != man.size() || cr.trailer != tr_stored ||
+      manifest_trailer(man.data(), man.size() - 8) != tr_stored || cr.group != g.id)
+    return fail(JITC_EINCOMPLETE, "jitc_restore: commit record does not match the manifest");
+  memcpy(&mv->h, man.data(), sizeof(ManifestHdr));
+  const ManifestHdr& h = mv->h;
+  if (h.magic != kMagicManifest || h.layout_hash != g.layout_hash || h.n_c != g.n_c || h.image_bytes != g.L ||
+      h.chunk_bytes != g.C || h.v_star != cr.v_star)
+    return fail(JITC_ELAYOUT, "jitc_restore: manifest layout differs from the registered tensors");
+  size_t q = sizeof(ManifestHdr);
+  mv->writers.resize(h.k);
+  memcpy(mv->writers.data(), man.data() + q, 4ull * h.k);
+  q = align_up(q + 4ull * h.k, 8);
+  size_t t0 = q;
+  for (uint32_t i = 0; i < h.n_tensors; ++i) {
+    uint16_t ln;
+    memcpy(&ln, man.data() + q, 2);
+    q += 2 + ln + 20;
+  }
+  q = t0 + align_up(q - t0, 8);
+  if (q + 8 * (h.n_c + 1) > man.size()) return fail(JITC_EINCOMPLETE, "jitc_restore: manifest truncated");
+  mv->d.resize(h.n_c);
+  memcpy(mv->d.data(), man.data() + q, 8 * h.n_c);
+  memcpy(&mv->root, man.data() + q + 8 * h.n_c, 8);
+  if (root_of(h.layout_hash, mv->d.data(), h.n_c) != mv->root)
+    return fail(JITC_EINCOMPLETE, "jitc_restore: manifest digests do not chain to its root");
+  return JITC_OK;
+}
+
+static jitc_status compare_digests(jitc_ctx* c, GroupState& g, const std::vector<uint64_t>& want, jitc_stats* stats) {
+  if (g.n_c) {
+    CU(cudaMemcpyAsync(c->h_dig, g.d_dig2, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
+    CU(cudaStreamSynchronize(c->s_comp));
+  }
+  for (uint64_t ch = 0; ch < g.n_c; ++ch)
+    if (c->h_dig[ch] != want[ch]) {
+      if (stats) stats->first_bad_chunk = (int32_t)ch;
+      return fail(JITC_ECORRUPT, "jitc_restore: group " + std::to_string(g.id) + " chunk " + std::to_string(ch) +
+                                     " does not match the checkpoint digest");
+    }
+  return JITC_OK;
+}
+
+// Executes a restore plan (jitc_plan.cc) round by round: H2D on the copy
+// stream; K2 packs, NCCL send/recv or all-gather and K3 unpacks on the
+// compute stream; slot reuse ordered by the ready/free events.
+static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<PlanOp>& ops, uint32_t S,
+                                jitc_stats* stats) {
+  if (S > (uint32_t)jitc_ctx::kSlots) return fail(JITC_EINVAL, "execute_plan: too many slots");
+  bool used[jitc_ctx::kSlots] = {false};
+  size_t i = 0;
+  uint32_t rounds = 0;
+  while (i < ops.size()) {
+    if (ops[i].kind == kOpDigestSend || ops[i].kind == kOpDigestRecv) {
+      ++i;
+      continue;
+    }
+    const uint32_t j = ops[i].round;
+    size_t e = i;
+    while (e < ops.size() && ops[e].round == j && ops[e].kind != kOpDigestSend && ops[e].kind != kOpDigestRecv) ++e;
+    const uint32_t sl = ops[i].slot;
+    ++rounds;
+    // 1. host -> device on the copy stream
+    bool any_h2d = false;
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpH2D) continue;
+      if (!any_h2d && used[sl]) CU(cudaStreamWaitEvent(c->s_copy, c->ev_free[sl], 0));
+      any_h2d = true;
+      CU(cudaMemcpyAsync(c->staging + op.off, g.img_h + op.a, op.bytes, cudaMemcpyHostToDevice, c->s_copy));
+      if (stats) stats->h2d_bytes += op.bytes;
+    }
+    if (any_h2d) {
+      CU(cudaEventRecord(c->ev_ready[sl], c->s_copy));
+      CU(cudaStreamWaitEvent(c->s_comp, c->ev_ready[sl], 0));
+    }
+    // 2. K2 packs (PEER writers)
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpPack) continue;
+      uint32_t lo, hi;
+      seg_span(g, op.a, op.b, &lo, &hi);
+      jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, c->staging + op.off, op.a), g.d_dig2, op.b - op.a);
+      if (st) return st;
+    }
+    // 3. NCCL: point-to-point (PEER) and all-gather (HOST, n > 1)
+    bool p2p = false;
+    for (size_t q = i; q < e; ++q) p2p |= ops[q].kind == kOpSend || ops[q].kind == kOpRecv;
+    if (p2p) {
+      NC(ncclGroupStart());
+      for (size_t q = i; q < e; ++q) {
+        const PlanOp& op = ops[q];
+        if (op.kind == kOpSend) NC(ncclSend(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+        if (op.kind == kOpRecv) NC(ncclRecv(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+        if (stats) stats->p2p_bytes += op.bytes;
+      }
+      NC(ncclGroupEnd());
+    }
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpAllGather) continue;
+      uint8_t* base = c->staging + op.off;
+      NC(ncclAllGather(base + (uint64_t)c->comm_rank * op.bytes, base, op.bytes, ncclUint8, c->comm, c->s_comp));
+      if (stats) stats->p2p_bytes += (uint64_t)(c->comm_n - 1) * op.bytes;
+    }
+    // 4. K3 unpack + verify of every block of the round (<= kMaxRanges per launch)
+    LaunchRanges lr{};
+    uint64_t bytes = 0;
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpUnpack) continue;
+      uint32_t lo, hi;
+      seg_span(g, op.a, op.b, &lo, &hi);
+      add_range(lr, lo, hi, c->staging + op.off, op.a);
+      bytes += op.b - op.a;
+      if (lr.n == kMaxRanges) {
+        jitc_status st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
+        if (st) return st;
+        lr = LaunchRanges{};
+        bytes = 0;
+      }
+    }
+    if (lr.n) {
+      jitc_status st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
+      if (st) return st;
+    }
+    CU(cudaEventRecord(c->ev_free[sl], c->s_comp));
+    used[sl] = true;
+    i = e;
+  }
+  if (stats) stats->rounds += rounds;
+  return JITC_OK;
+}
+
+static jitc_status make_plan(jitc_ctx* c, const PlanInput& in, std::vector<PlanOp>* ops, uint32_t* S) {
+  uint64_t R;
+  std::string why;
+  if (!build_restore_plan(in, ops, &R, S, &why)) return fail(JITC_ENOMEM, "jitc_restore: " + why);
+  return JITC_OK;
+}
+
+// HOST mode: this rank (or, with a communicator, every comm rank) loads a
+// 1/n slice of the committed image H2D; slices are all-gathered over NVLink
+// round by round and every round is unpacked+verified by K3.
+static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
+  ManifestView mv;
+  jitc_status st = load_manifest(c, g, &mv);
+  if (st) return st;
+  if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
+  const int n = c->comm ? c->comm_n : 1;
+  if (n > 1 && !g.img_shm)
+    return fail(JITC_EINVAL, "jitc_restore: HOST mode across ranks needs a shared image_dir (use PEER mode)");
+  if (n == 1 && (c->cfg.flags & JITC_F_ZERO_COPY_H2D)) {
+    st = run_segments(c, g, kUnpack, one_range(0, (uint32_t)g.segs.size(), g.img_d, 0), g.d_dig2, g.L);
+    if (st) return st;
+    if (stats) stats->rounds += 1, stats->h2d_bytes += g.L;
+  } else {
+    PlanInput in;
+    in.mode = JITC_RESTORE_HOST;
+    in.n_c = g.n_c;
+    in.chunk_bytes = g.C;
+    in.image_bytes = g.L;
+    in.n = n;
+    in.me = c->comm ? c->comm_rank : 0;
+    in.staging_bytes = c->staging_bytes;
+    in.slot_bytes = c->slot_bytes;
+    if (c->comm) {
+      for (int32_t m : g.members) {
+        int r = comm_rank_of(c, m);
+        if (r >= 0) in.participants.push_back(r);
+      }
+      std::sort(in.participants.begin(), in.participants.end());
+    } else {
+      in.participants = {0};
+    }
+    std::vector<PlanOp> ops;
+    uint32_t S = 0;
+    st = make_plan(c, in, &ops, &S);
+    if (st) return st;
+    st = execute_plan(c, g, ops, S, stats);
+    if (st) return st;
+  }
+  st = compare_digests(c, g, mv.d, stats);
+  if (st) return st;
+  g.man_d = mv.d;
+  g.man_root = mv.root;
+  g.has_man = true;
+  if (stats) stats->image_bytes += g.L;
+  return JITC_OK;
+}
+
+// PEER mode: the selection's writers pack their O5 ranges from live HBM (K2)
+// and send them over NVLink to every member that is not a writer; receivers
+// unpack+verify (K3) against the writers' digests (broadcast first).
+static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection& gs, jitc_stats* stats) {
+  if (!c->comm) return fail(JITC_ESTATE, "jitc_restore: PEER mode needs a communicator");
+  if (gs.writers.empty()) return JITC_OK;  // dropped OPTIONAL group
+  if (gs.layout_hash != g.layout_hash || gs.n_c != g.n_c || gs.image_bytes != g.L)
+    return fail(JITC_ELAYOUT, "jitc_restore: selection layout differs from the registered one");
+  PlanInput in;
+  in.mode = JITC_RESTORE_PEER;
+  in.n_c = g.n_c;
+  in.chunk_bytes = g.C;
+  in.image_bytes = g.L;
+  in.n = c->comm_n;
+  in.me = c->comm_rank;
+  in.staging_bytes = c->staging_bytes;
+  in.slot_bytes = c->slot_bytes;
+  for (int32_t w : gs.writers) {
+    int r = comm_rank_of(c, w);
+    if (r < 0) return fail(JITC_EINVAL, "jitc_restore: a writer is not in the communicator");
+    in.writers.push_back(r);
+  }
+  for (int32_t m : gs.members) {
+    if (std::find(gs.writers.begin(), gs.writers.end(), m) != gs.writers.end()) continue;
+    int r = comm_rank_of(c, m);
+    if (r >= 0) in.dests.push_back(r);
+  }
+  const int my_s = (int)(std::find(in.writers.begin(), in.writers.end(), in.me) - in.writers.begin());
+  const bool is_writer = my_s < (int)in.writers.size();
+  const bool is_dst = std::find(in.dests.begin(), in.dests.end(), in.me) != in.dests.end();
+  std::vector<PlanOp> ops;
+  uint32_t S = 0;
+  jitc_status st = make_plan(c, in, &ops, &S);
+  if (st) return st;
+  if (!is_writer && !is_dst) return JITC_OK;
+  // 1. the lowest writer sends the selected class's digests to every destination
+  uint64_t* d_expect = g.d_dig;
+  if (is_writer && (!g.has_fp || g.fp_root != gs.root))
+    return fail(JITC_ESTATE, "jitc_restore: writer fingerprint differs from the selected class");
+  if (is_writer && my_s == 0 && g.n_c)
+    CU(cudaMemcpyAsync(d_expect, g.fp.data(), g.n_c * 8, cudaMemcpyHostToDevice, c->s_comp));
+  bool any = false;
+  for (const PlanOp& op : ops) any |= op.kind == kOpDigestSend || op.kind == kOpDigestRecv;
+  if (any && g.n_c) {
+    NC(ncclGroupStart());
+    for (const PlanOp& op : ops) {
+      if (op.kind == kOpDigestSend) NC(ncclSend(d_expect, g.n_c, ncclUint64, op.peer, c->comm, c->s_comp));
+      if (op.kind == kOpDigestRecv) NC(ncclRecv(d_expect, g.n_c, ncclUint64, op.peer, c->comm, c->s_comp));
+    }
+    NC(ncclGroupEnd());
+  }
+  std::vector<uint64_t> want(g.n_c);
+  if (is_dst) {
+    if (g.n_c) CU(cudaMemcpyAsync(want.data(), d_expect, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
+    CU(cudaStreamSynchronize(c->s_comp));
+    if (root_of(g.layout_hash, want.data(), g.n_c) != gs.root)
+      return fail(JITC_ECORRUPT, "jitc_restore: received digests do not chain to the selected root");
+  } else {
+    want = g.fp;
+  }
+  if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
+  // 2. data rounds
+  st = execute_plan(c, g, ops, S, stats);
+  if (st) return st;
+  CU(cudaStreamSynchronize(c->s_comp));
+  if (is_dst) {
+    st = compare_digests(c, g, want, stats);
+    if (st) return st;
+    g.man_d = want;
+    g.man_root = gs.root;
+    g.has_man = true;
+    if (stats) stats->image_bytes += g.L;
+  } else if (g.n_c) {  // the writer's re-digest of its own range must still match
+    CU(cudaMemcpyAsync(c->h_dig, g.d_dig2, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
+    CU(cudaStreamSynchronize(c->s_comp));
+    uint64_t c0, c1;
+    shard_range(g.n_c, in.writers.size(), my_s, &c0, &c1);
+    for (uint64_t ch = c0; ch < c1; ++ch)
+      if (c->h_dig[ch] != want[ch]) return fail(JITC_EUNSTABLE, "jitc_restore: writer state changed");
+  }
+  return JITC_OK;
+}
+
+jitc_status jitc_restore(jitc_ctx* c, uint32_t group, int32_t mode, const void* selection, size_t sel_len,
+                         jitc_stats* stats) {
+  if (!c) return fail(JITC_EINVAL, "jitc_restore: null ctx");
+  if (mode != JITC_RESTORE_HOST && mode != JITC_RESTORE_PEER) return fail(JITC_EINVAL, "jitc_restore: bad mode");
+  Selection sel;
+  bool have_sel = false;
+  if (selection) {
+    std::string why;
+    if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
+      return fail(JITC_EINVAL, "jitc_restore: " + why);
+    if (sel.status != JITC_OK) return fail(sel.status, "jitc_restore: selection status is not OK");
+    have_sel = true;
+  } else if (mode == JITC_RESTORE_PEER) {
+    return fail(JITC_EINVAL, "jitc_restore: PEER mode needs the selection");
+  }
+  CU(cudaSetDevice(c->device));
+  if (stats) memset(stats, 0, sizeof *stats), stats->first_bad_chunk = -1;
+  CallTimer t(c);
+  CU(cudaEventRecord(c->ev_t0, c->s_comp));
+  for (auto& kv : c->groups) {
+    GroupState& g = kv.second;
+    if (!g.held || (group != JITC_ALL_GROUPS && g.id != group)) continue;
+    const GroupSelection* gs = have_sel ? sel.find(g.id) : nullptr;
+    if (have_sel && !gs) return fail(JITC_ELAYOUT, "jitc_restore: group missing from selection");
+    if (gs && gs->writers.empty()) continue;  // dropped OPTIONAL group: nothing to restore
+    jitc_status st = mode == JITC_RESTORE_HOST ? restore_host(c, g, stats) : restore_peer(c, g, *gs, stats);
+    if (st) {
+      harvest(c);
+      return st;
+    }
+  }
+  CU(cudaEventRecord(c->ev_t1, c->s_comp));
+  CU(cudaEventSynchronize(c->ev_t1));
+  finish_stats(c, t, stats, true);
+  return JITC_OK;
+}
+
+// ------------------------------------------------------------ verify (A12)
+jitc_status jitc_verify(jitc_ctx* c, uint32_t group, const void* expected, size_t len, uint64_t* first_bad) {
+  if (!c) return fail(JITC_EINVAL, "jitc_verify: null ctx");
+  if (first_bad) *first_bad = UINT64_MAX;
+  auto it = c->groups.find(group);
+  if (it == c->groups.end() || !it->second.held) return fail(JITC_EINVAL, "jitc_verify: group not registered");
+  GroupState& g = it->second;
+  std::vector<uint64_t> want;
+  if (expected) {
+    std::vector<BlobView> bv;
+    std::string why;
+    if (!parse_blobs(static_cast<const uint8_t*>(expected), len, &bv, &why)) return fail(JITC_EINVAL, "jitc_verify: " + why);
+    const RecordView* rv = nullptr;
+    for (auto& b : bv)
+      for (auto& r : b.recs)
+        if (r.h.group == group && !rv) rv = &r;
+    if (!rv) return fail(JITC_EINVAL, "jitc_verify: expected blob has no record of the group");
+    if (rv->h.layout_hash != g.layout_hash || rv->h.n_c != g.n_c) return fail(JITC_ELAYOUT, "jitc_verify: layout differs");
+    want.assign(rv->d, rv->d + rv->h.n_c);
+  } else {
+    if (!g.has_man) return fail(JITC_ESTATE, "jitc_verify: no manifest (restore or commit first)");
+    want = g.man_d;
+  }
+  CU(cudaSetDevice(c->device));
+  CallTimer t(c);
+  if (g.n_c) {
+    CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
+    jitc_status st = run_segments(c, g, kDigest, one_range(0, (uint32_t)g.segs.size(), nullptr, 0), g.d_dig2, g.L);
+    if (st) return st;
+    CU(cudaMemcpyAsync(c->h_dig, g.d_dig2, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
+  }
+  CU(cudaStreamSynchronize(c->s_comp));
+  harvest(c);
+  for (uint64_t ch = 0; ch < g.n_c; ++ch)
+    if (c->h_dig[ch] != want[ch]) {
+      if (first_bad) *first_bad = ch;
+      return fail(JITC_ECORRUPT, "jitc_verify: chunk " + std::to_string(ch) + " differs");
+    }
+  return JITC_OK;
+}
+

@@ -1,0 +1,121 @@
+// libjitc.so hang detection (NEXT-1): event watch-list + native watchdog
+// thread (§3.1-3.2).
+#include "jitc_ctx.h"
+
+using namespace jitc;
+
+// ------------------------------------------------------------ watchdog (NEXT-1)
+// PAPER.md:124-126 §3.1: events recorded after collectives are put on a
+// watch-list; a watchdog thread polls them with cudaEventQuery and treats
+// one that stays incomplete past a timeout as a hang of the collective.
+// PAPER.md:132-134 §3.2: the checkpoint is then taken on a side stream by the
+// watchdog thread itself -- here entirely in C++ (no Python callback, so the
+// GIL cannot block it) on the library's non-blocking streams.
+
+static void watchdog_loop(jitc_ctx* c) {
+  cudaSetDevice(c->device);
+  const double t0 = now_ms();
+  for (;;) {
+    std::unique_lock<std::mutex> lk(c->wmu);
+    if (!c->wrun) return;
+    double now = now_ms();
+    bool hang = false;
+    for (size_t i = 0; i < c->watches.size();) {
+      cudaError_t q = cudaEventQuery(c->watches[i].ev);
+      if (q == cudaSuccess) {
+        c->watches.erase(c->watches.begin() + i);
+        continue;
+      }
+      if (q != cudaErrorNotReady) cudaGetLastError();
+      if (now - c->watches[i].t_added >= c->timeout_ms) {
+        hang = true;
+        c->fired_tag = c->watches[i].tag;
+        c->waited_ms = now - c->watches[i].t_added;
+        break;
+      }
+      ++i;
+    }
+    if (hang) {
+      c->fired = true;
+      c->detect_ms = now - t0;
+      lk.unlock();
+      double ta = now_ms();
+      if (c->action == JITC_ON_HANG_LOCAL_CAPTURE) {
+        jitc_stats st{};
+        jitc_status r = local_capture(c, &st);
+        lk.lock();
+        c->action_status = r;
+        c->action_stats = st;
+        lk.unlock();
+      }
+      if (c->hang_fn) c->hang_fn(c->hang_user, c->fired_tag, c->waited_ms);
+      lk.lock();
+      c->action_ms = now_ms() - ta;
+      c->action_done = true;
+      c->wrun = false;
+      c->wcv.notify_all();
+      return;
+    }
+    c->wcv.wait_for(lk, std::chrono::microseconds(200));
+  }
+}
+
+static void stop_thread(jitc_ctx* c) {
+  {
+    std::lock_guard<std::mutex> lk(c->wmu);
+    c->wrun = false;
+    c->wcv.notify_all();
+  }
+  if (c->wthread.joinable()) c->wthread.join();
+}
+
+
+jitc_status jitc_watch_event(jitc_ctx* c, void* event, uint64_t tag) {
+  if (!c || !event) return fail(JITC_EINVAL, "jitc_watch_event: null argument");
+  std::lock_guard<std::mutex> lk(c->wmu);
+  c->watches.push_back({(cudaEvent_t)event, tag, now_ms()});
+  return JITC_OK;
+}
+
+jitc_status jitc_watchdog_start(jitc_ctx* c, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user) {
+  if (!c) return fail(JITC_EINVAL, "jitc_watchdog_start: null ctx");
+  if (action != JITC_ON_HANG_NOTIFY && action != JITC_ON_HANG_LOCAL_CAPTURE)
+    return fail(JITC_EINVAL, "jitc_watchdog_start: bad action");
+  stop_thread(c);  // a previous watchdog; the watch-list is kept
+  std::lock_guard<std::mutex> lk(c->wmu);
+  c->timeout_ms = timeout_ms;
+  c->action = action;
+  c->hang_fn = fn;
+  c->hang_user = user;
+  c->fired = c->action_done = false;
+  c->action_status = JITC_OK;
+  c->action_stats = jitc_stats{};
+  c->action_stats.first_bad_chunk = -1;
+  c->wrun = true;
+  c->wthread = std::thread(watchdog_loop, c);
+  return JITC_OK;
+}
+
+jitc_status jitc_watchdog_wait(jitc_ctx* c, uint32_t max_ms, int32_t* fired, uint64_t* tag, double* waited_ms,
+                               double* action_ms, jitc_stats* action_stats) {
+  if (!c || !fired) return fail(JITC_EINVAL, "jitc_watchdog_wait: null argument");
+  std::unique_lock<std::mutex> lk(c->wmu);
+  c->wcv.wait_for(lk, std::chrono::milliseconds(max_ms), [c] { return c->action_done; });
+  *fired = c->action_done ? 1 : 0;
+  if (tag) *tag = c->fired_tag;
+  if (waited_ms) *waited_ms = c->waited_ms;
+  if (action_ms) *action_ms = c->action_ms;
+  if (action_stats) *action_stats = c->action_stats;
+  jitc_status st = c->action_done ? c->action_status : JITC_OK;
+  if (st) set_error("jitc_watchdog_wait: the on-hang capture failed with status " + std::to_string(st));
+  return st;
+}
+
+jitc_status jitc_watchdog_stop(jitc_ctx* c) {
+  if (!c) return fail(JITC_EINVAL, "jitc_watchdog_stop: null ctx");
+  stop_thread(c);
+  std::lock_guard<std::mutex> lk(c->wmu);
+  c->watches.clear();
+  return JITC_OK;
+}
+
