@@ -262,9 +262,29 @@ def run_jitc(args):
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms_step, ms_step_wall = tt.tolist()
 
+    # robustness variant: one more step while an emulated
+    # hung collective (32 spinning CTAs on another stream) occupies the GPU,
+    # as when a NCCL kernel waits forever on a dead peer
+    under_hang = None
+    if args.hang_ctas > 0:
+        kc_keep = {k: ctx.kernel_counters(k) for k in (J.K_DIGEST, J.K_PACK, J.K_UNPACK)}
+        hs = torch.cuda.Stream()
+        J.inject_hang(hs.cuda_stream, args.hang_ctas, slot=5)
+        try:
+            t0 = time.perf_counter()
+            cap_h, res_h, _ = step(False)
+            dt = time.perf_counter() - t0
+        finally:
+            J.inject_release(5)
+        hs.synchronize()
+        under_hang = {"hung_ctas": args.hang_ctas, "step_s": round(dt, 4),
+                      "value_GBps": round(L_total / dt / 1e9, 3),
+                      "capture_GBps": round(cap_h["image_bytes"] / (cap_h["ms_host"] * 1e-3) / 1e9, 3),
+                      "restore_GBps": round(res_h["image_bytes"] / (res_h["ms_host"] * 1e-3) / 1e9, 3)}
+
     # roofline of the dominant kernel (largest total time in the timed region)
     kinds = {J.K_DIGEST: "K1_digest", J.K_PACK: "K2_pack_digest", J.K_UNPACK: "K3_unpack_verify"}
-    kc = {k: ctx.kernel_counters(k) for k in kinds}
+    kc = kc_keep if under_hang is not None else {k: ctx.kernel_counters(k) for k in kinds}
     dom = max(kc, key=lambda k: kc[k]["ms"])
     c = kc[dom]
     rw = 1 if dom == J.K_DIGEST else 2          # K1 reads L; K2/K3 read L and write L
@@ -313,6 +333,7 @@ def run_jitc(args):
                     "d2h_bytes_per_step": L_total // world + rec_bytes,
                     "note": "host wall clock around the public Python API step (ctypes, manifest file I/O included)"},
             "gpu_launches": launches[0],
+            "under_hang": under_hang,
             "clocks": clk.summary(),
         }
         if not args.no_cpu_baseline:
@@ -337,6 +358,7 @@ def main():
     ap.add_argument("--zero-copy", action="store_true")
     ap.add_argument("--image-dir", default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
     ap.add_argument("--ref-sample", type=int, default=1024, help="MiB per reference step")
     args = ap.parse_args()
     if args.warmup < 3:
