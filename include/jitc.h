@@ -135,7 +135,7 @@ typedef struct {
 } jitc_stats;
 
 /* Cumulative per-kernel counters (bench roofline): kind 1 = K1 digest,
- * 2 = K2 pack+digest, 3 = K3 unpack+verify. */
+ * 2 = K2 pack+digest, 3 = K3 unpack+verify, 4 = K5 peer pull+verify. */
 typedef struct {
     uint64_t launches;
     uint64_t bytes;            /* algorithmic image bytes processed                            */
@@ -249,6 +249,19 @@ jitc_status jitc_capture_local(jitc_ctx* ctx, jitc_stats* stats);
  * digests.  selection may be NULL in HOST mode (taken from the manifest). */
 jitc_status jitc_restore(jitc_ctx* ctx, uint32_t group, int32_t mode, const void* selection,
                          size_t sel_len, jitc_stats* stats);
+/* F1 fusion -- intra-node PEER restore by direct peer-memory reads (no NCCL,
+ * no staging).  A writer (after jitc_fingerprint, while its state stays
+ * quiesced) publishes CUDA IPC handles of the allocations holding its
+ * registered tensors and its digests into image_dir (g<group>.peer.<rank>).
+ * The replacement maps every selected writer's export and ONE kernel (K5)
+ * reads writer s's chunk range O5(n_c, k, s) over NVLink, scatters it into
+ * its own tensors and re-digests it in the same pass; digests that differ
+ * from the writers' => JITC_ECORRUPT (stats->first_bad_chunk).  The mappings
+ * are closed before returning, after which the writers may resume.  Not for
+ * VMM / expandable-segment allocations (not IPC-exportable: JITC_ECUDA). */
+jitc_status jitc_peer_export(jitc_ctx* ctx, uint32_t group);
+jitc_status jitc_restore_pull(jitc_ctx* ctx, uint32_t group, const void* selection, size_t sel_len,
+                              jitc_stats* stats);
 /* A12: K1 over the live tensors of `group`, compared with `expected` (a
  * record blob holding that group) or, if NULL, with the manifest digests of
  * the last restore / commit.  Mismatch => JITC_ECORRUPT, *first_bad_chunk

@@ -198,6 +198,7 @@ jitc_status jitc_register(jitc_ctx* c, uint32_t group, int32_t policy, const int
   g.n_c = (g.L + g.C - 1) / g.C;
   // segment table: pieces <= kMaxSegBytes that never cross a chunk boundary
   g.segs.clear();
+  g.seg_tensor.clear();
   for (size_t i = 0; i < n; ++i) {
     uint64_t nb = t[i].nbytes, base = (uint64_t)t[i].ptr;
     uint64_t end_img = align_up(g.off[i] + nb, kAlign);
@@ -214,6 +215,7 @@ jitc_status jitc_register(jitc_ctx* c, uint32_t group, int32_t policy, const int
       s.chunk = (uint32_t)(img / g.C);
       s.flags = ((s.src % 16) == 0 ? kSegAligned16 : 0u) | ((s.src % 8) == 0 ? kSegAligned8 : 0u);
       g.segs.push_back(s);
+      g.seg_tensor.push_back((uint32_t)i);
       p += len;
     }
   }
@@ -223,6 +225,8 @@ jitc_status jitc_register(jitc_ctx* c, uint32_t group, int32_t policy, const int
     CU(cudaMemcpyAsync(g.d_segs, g.segs.data(), g.segs.size() * sizeof(Seg), cudaMemcpyHostToDevice, c->s_comp));
   CU(cudaMalloc(&g.d_dig, std::max<uint64_t>(g.n_c, 1) * 8));
   CU(cudaMalloc(&g.d_dig2, std::max<uint64_t>(g.n_c, 1) * 8));
+  CU(cudaMalloc(&g.d_remote, std::max<size_t>(g.segs.size(), 1) * 8));
+  g.h_remote.assign(g.segs.size(), 0);
   CU(cudaStreamSynchronize(c->s_comp));
   st = ensure_h_dig(c, g.n_c);
   if (st) return st;
@@ -444,7 +448,7 @@ jitc_status jitc_exchange_records(jitc_ctx* c, const void* mine, size_t len, voi
 
 // ------------------------------------------------------------ counters
 jitc_status jitc_kernel_counters(jitc_ctx* c, int32_t kind, jitc_kernel_counter* out) {
-  if (!c || !out || kind < 1 || kind > 3) return fail(JITC_EINVAL, "jitc_kernel_counters: bad argument");
+  if (!c || !out || kind < 1 || kind > 4) return fail(JITC_EINVAL, "jitc_kernel_counters: bad argument");
   *out = c->kc[kind];
   return JITC_OK;
 }

@@ -41,7 +41,10 @@ struct GroupState {
   std::vector<uint64_t> off;
   uint64_t C = 0, L = 0, n_c = 0, layout_hash = 0;
   std::vector<Seg> segs;
+  std::vector<uint32_t> seg_tensor;  // tensor index of every segment
   Seg* d_segs = nullptr;
+  uint64_t* d_remote = nullptr;      // K5: per-segment peer source address
+  std::vector<uint64_t> h_remote;
   uint64_t* d_dig = nullptr;   // K1 digests
   uint64_t* d_dig2 = nullptr;  // K2 / K3 digests
   // last fingerprint
@@ -122,7 +125,7 @@ struct jitc_ctx {
   jitc_status action_status = JITC_OK;
   jitc_stats action_stats{};
   // counters
-  jitc_kernel_counter kc[4]{};
+  jitc_kernel_counter kc[5]{};
   uint64_t launches_in_call = 0;
   double kernel_ms_in_call = 0;
 };
@@ -164,10 +167,10 @@ struct CallTimer {
 
 // Kernel launch with optional event bracketing (JITC_F_TIME_KERNELS).
 inline jitc_status run_segments(jitc_ctx* c, GroupState& g, int mode, const LaunchRanges& r, uint64_t* dig,
-                         uint64_t bytes) {
+                         uint64_t bytes, const uint64_t* remote = nullptr) {
   bool timed = (c->cfg.flags & JITC_F_TIME_KERNELS) && c->kev_used + 2 <= c->kev.size();
   if (timed) CU(cudaEventRecord(c->kev[c->kev_used], c->s_comp));
-  CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->d_work, c->s_comp));
+  CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->d_work, c->s_comp, remote));
   if (timed) {
     CU(cudaEventRecord(c->kev[c->kev_used + 1], c->s_comp));
     c->kev_kind[c->kev_used / 2] = mode;
@@ -247,6 +250,8 @@ inline void free_group(GroupState& g) {
   if (g.d_segs) cudaFree(g.d_segs);
   if (g.d_dig) cudaFree(g.d_dig);
   if (g.d_dig2) cudaFree(g.d_dig2);
+  if (g.d_remote) cudaFree(g.d_remote);
+  g.d_remote = nullptr;
   if (g.img_h) {
     if (g.img_shm) {
       cudaHostUnregister(g.img_h);
@@ -314,4 +319,6 @@ jitc_status commit_impl(jitc_ctx* c, const void* selection, size_t sel_len, bool
 jitc_status local_capture(jitc_ctx* c, jitc_stats* st);
 // defined in jitc_ctx.cc
 jitc_status fingerprint_group(jitc_ctx* c, GroupState& g);
+// defined in jitc_restore.cc: K2/K3/K5 digests of the group vs `want` (ECORRUPT + first bad chunk)
+jitc_status compare_digests(jitc_ctx* c, GroupState& g, const std::vector<uint64_t>& want, jitc_stats* stats);
 }  // namespace jitc

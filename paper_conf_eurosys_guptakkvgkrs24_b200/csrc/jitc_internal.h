@@ -54,7 +54,7 @@ struct Seg {
 enum : uint32_t { kSegAligned16 = 1u, kSegAligned8 = 2u };
 static_assert(sizeof(Seg) == 32, "Seg must be 32 bytes");
 
-enum KernelMode : int { kDigest = 1, kPack = 2, kUnpack = 3 };
+enum KernelMode : int { kDigest = 1, kPack = 2, kUnpack = 3, kPull = 4 };  // kPull: F1 fused peer pull
 
 // A launch covers up to kMaxRanges segment ranges; range r reads/writes the
 // image bytes through `base[r]`, which corresponds to image offset base_off[r].
@@ -71,8 +71,9 @@ struct LaunchRanges {
 // kernels (jitc_kernels.cu)
 // d_work: 2 x u32 zero-initialised device counters, private to the stream
 // (the kernel resets them when it finishes).
+// d_remote (kPull only): per-segment source address in a peer's memory.
 cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig,
-                            int grid, uint32_t* d_work, cudaStream_t s);
+                            int grid, uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote = nullptr);
 cudaError_t launch_phase_write(uint64_t* dev_slot, uint64_t value, cudaStream_t s);
 int segment_grid(int device);
 cudaError_t device_check(int device, std::string* why);

@@ -5,6 +5,10 @@
 //                     HBM, or mapped pinned host memory), JF64 in the same pass
 //  K3 unpack+verify : image bytes (staging slot / mapped host) -> scatter into
 //                     the tensors, JF64 of the bytes read
+//  K5 pull+verify   : (F1 fusion) the writers' tensors read directly over
+//                     NVLink through CUDA IPC mappings -> the local tensors,
+//                     JF64 in the same pass: transfer and verification in one
+//                     kernel, no staging and no writer-side kernel
 //  K4 (harness)     : counter-based synthetic state, optimizer-update and
 //                     bit-flip injectors
 //
@@ -117,7 +121,8 @@ constexpr uint32_t kBatch = 8;
 template <int MODE>
 __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ segs, LaunchRanges R,
                                                        unsigned long long* __restrict__ dig,
-                                                       unsigned int* __restrict__ work) {
+                                                       unsigned int* __restrict__ work,
+                                                       const uint64_t* __restrict__ remote) {
   const uint32_t total = R.prefix[R.n];
   const uint32_t nbatch = (total + kBatch - 1) / kBatch;
   const int tid = threadIdx.x;
@@ -147,18 +152,23 @@ __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ s
       const uint64_t rel = sg.img_off - R.base_off[r];
       uint8_t* img = reinterpret_cast<uint8_t*>(R.base[r]) + rel;  // 16-B aligned (staging / host image)
       uint8_t* ten = reinterpret_cast<uint8_t*>(sg.src);
+      // kPull: the same bytes in a peer's tensor, read over NVLink (CUDA IPC mapping)
+      const uint8_t* peer = MODE == kPull ? reinterpret_cast<const uint8_t*>(remote[R.seg_begin[r] + (v - R.prefix[r])])
+                                          : nullptr;
       const uint64_t data = sg.data_bytes;
       const uint64_t words = (data + sg.pad_bytes) >> 3;
       const uint64_t g0 = sg.img_off >> 3;
       uint64_t body_words = 0;
+      const bool vec = MODE == kPull ? (((uint64_t)peer | sg.src) & 15) == 0 : (sg.flags & kSegAligned16) != 0;
 
-      if (sg.flags & kSegAligned16) {
+      if (vec) {
         const uint32_t nvec = (uint32_t)(data >> 4);
         body_words = 2ull * nvec;
         const uint4* in = MODE == kUnpack ? reinterpret_cast<const uint4*>(img)
+                        : MODE == kPull   ? reinterpret_cast<const uint4*>(peer)
                                           : reinterpret_cast<const uint4*>(ten);
         uint4* out = MODE == kPack ? reinterpret_cast<uint4*>(img)
-                   : MODE == kUnpack ? reinterpret_cast<uint4*>(ten) : nullptr;
+                   : (MODE == kUnpack || MODE == kPull) ? reinterpret_cast<uint4*>(ten) : nullptr;
         uint32_t i = tid;
         // key of word 2i is (g0 + 2i + 1) * PHI; the step between a thread's
         // consecutive vectors is 2 * kThreads words.
@@ -187,12 +197,15 @@ __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ s
       }
       // Remaining words: unaligned tensors (all of them), the < 16-byte data
       // tail, and the zero padding that closes the tensor's image slot.
-      const bool al8 = (sg.flags & kSegAligned8) != 0;
+      const bool al8 = MODE == kPull ? (((uint64_t)peer | sg.src) & 7) == 0 : (sg.flags & kSegAligned8) != 0;
       for (uint64_t w = body_words + tid; w < words; w += kThreads) {
         const uint64_t b = 8 * w;
         uint64_t x;
         if (MODE == kUnpack) {
           x = *reinterpret_cast<const uint64_t*>(img + b);
+          if (b < data) store_word_bytes(ten, b, data, x, al8);
+        } else if (MODE == kPull) {
+          x = load_word_bytes(peer, b, data, al8);
           if (b < data) store_word_bytes(ten, b, data, x, al8);
         } else {
           x = load_word_bytes(ten, b, data, al8);
@@ -320,7 +333,8 @@ int segment_grid(int device) {
 cudaError_t preload_kernels() {
   cudaFuncAttributes fa;
   const void* fns[] = {(const void*)seg_kernel<kDigest>, (const void*)seg_kernel<kPack>,
-                       (const void*)seg_kernel<kUnpack>, (const void*)phase_write_kernel,
+                       (const void*)seg_kernel<kUnpack>, (const void*)seg_kernel<kPull>,
+                       (const void*)phase_write_kernel,
                        (const void*)gen_kernel, (const void*)update_kernel, (const void*)rne_kernel,
                        (const void*)bitflip_kernel, (const void*)hang_kernel, (const void*)release_kernel};
   for (const void* f : fns) {
@@ -348,16 +362,20 @@ cudaError_t device_check(int device, std::string* why) {
 }
 
 cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig, int grid,
-                            uint32_t* d_work, cudaStream_t s) {
+                            uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote) {
   uint32_t total = r.prefix[r.n];
   if (total == 0) return cudaSuccess;
   uint32_t nbatch = (total + kBatch - 1) / kBatch;
   int g = (int)(nbatch < (uint32_t)grid ? nbatch : (uint32_t)grid);
   auto* dig = reinterpret_cast<unsigned long long*>(d_dig);
   switch (mode) {
-    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work); break;
-    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work); break;
-    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work); break;
+    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr); break;
+    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr); break;
+    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr); break;
+    case kPull:
+      if (!d_remote) return cudaErrorInvalidValue;
+      seg_kernel<kPull><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, d_remote);
+      break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();

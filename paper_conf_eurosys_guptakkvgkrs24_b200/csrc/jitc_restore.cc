@@ -56,7 +56,7 @@ static jitc_status load_manifest(jitc_ctx* c, GroupState& g, ManifestView* mv) {
   return JITC_OK;
 }
 
-static jitc_status compare_digests(jitc_ctx* c, GroupState& g, const std::vector<uint64_t>& want, jitc_stats* stats) {
+jitc_status jitc::compare_digests(jitc_ctx* c, GroupState& g, const std::vector<uint64_t>& want, jitc_stats* stats) {
   if (g.n_c) {
     CU(cudaMemcpyAsync(c->h_dig, g.d_dig2, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
     CU(cudaStreamSynchronize(c->s_comp));

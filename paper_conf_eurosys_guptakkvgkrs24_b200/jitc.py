@@ -27,7 +27,7 @@ REQUIRED, OPTIONAL = 0, 1
 HOST, PEER = 0, 1
 ALL_GROUPS = 0xFFFFFFFF
 F_ZERO_COPY_D2H, F_ZERO_COPY_H2D, F_TIME_KERNELS, F_NO_SHM_UNLINK = 1, 2, 4, 8
-K_DIGEST, K_PACK, K_UNPACK = 1, 2, 3
+K_DIGEST, K_PACK, K_UNPACK, K_PULL = 1, 2, 3, 4
 
 
 class JitcError(RuntimeError):
@@ -110,6 +110,8 @@ def lib() -> ctypes.CDLL:
         "jitc_inject_release": ([u32], i32),
         "jitc_watch_event": ([vp, vp, u64], i32),
         "jitc_capture_local": ([vp, P(Stats)], i32),
+        "jitc_peer_export": ([vp, u32], i32),
+        "jitc_restore_pull": ([vp, u32, vp, sz, P(Stats)], i32),
         "jitc_persist": ([vp, u32, ctypes.c_char_p, P(Stats)], i32),
         "jitc_stage_in": ([vp, u32, ctypes.c_char_p, P(Stats)], i32),
         "jitc_waste_model": ([i32] + [ctypes.c_double] * 7 + [P(ctypes.c_double)] * 3, i32),
@@ -131,7 +133,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
-            "jitc_inject_release", "jitc_capture_local", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
+            "jitc_inject_release", "jitc_capture_local", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE = 0, 1
 
@@ -378,6 +380,15 @@ class Context:
         st = Stats()
         r = self._L.jitc_restore(self._h, group, mode, selection, len(selection) if selection else 0, ctypes.byref(st))
         _check(r, "jitc_restore", st.first_bad_chunk)
+        return st.as_dict()
+
+    def peer_export(self, group: int):
+        _check(self._L.jitc_peer_export(self._h, group), "jitc_peer_export")
+
+    def restore_pull(self, group: int, selection: bytes) -> dict:
+        st = Stats()
+        r = self._L.jitc_restore_pull(self._h, group, selection, len(selection), ctypes.byref(st))
+        _check(r, "jitc_restore_pull", st.first_bad_chunk)
         return st.as_dict()
 
     def verify(self, group: int, expected: Optional[bytes] = None) -> int:
