@@ -237,15 +237,31 @@ jitc_status jitc_register(jitc_ctx* c, uint32_t group, int32_t policy, const int
     g.img_path = gpath(c, group, ".img");
     int fd = open(g.img_path.c_str(), O_RDWR | O_CREAT, 0600);
     if (fd < 0) return fail(JITC_EIO, "jitc_register: open " + g.img_path + ": " + strerror(errno));
+    // Several ranks of a box register the same image.  Concurrent
+    // cudaHostRegister calls that fault the same fresh tmpfs pages in fail
+    // (error 304, measured with >= 8 GiB images: tools/pin_probe2.py), so
+    // the pages are allocated up front (posix_fallocate, idempotent) and the
+    // registration itself is serialised with an exclusive flock on the file.
+    flock(fd, LOCK_EX);
     struct stat sb;
-    if (fstat(fd, &sb) != 0 || ((uint64_t)sb.st_size != g.img_bytes && ftruncate(fd, (off_t)g.img_bytes) != 0)) {
+    int err = 0;
+    if (fstat(fd, &sb) != 0 || ((uint64_t)sb.st_size != g.img_bytes && ftruncate(fd, (off_t)g.img_bytes) != 0))
+      err = errno ? errno : EIO;
+    if (!err) err = posix_fallocate(fd, 0, (off_t)g.img_bytes);
+    if (err) {
+      flock(fd, LOCK_UN);
       close(fd);
-      return fail(JITC_EIO, "jitc_register: size " + g.img_path + ": " + strerror(errno));
+      return fail(JITC_EIO, "jitc_register: sizing " + g.img_path + ": " + strerror(err));
     }
     void* p = mmap(nullptr, g.img_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
-    close(fd);
-    if (p == MAP_FAILED) return fail(JITC_EIO, "jitc_register: mmap " + g.img_path + ": " + strerror(errno));
+    if (p == MAP_FAILED) {
+      flock(fd, LOCK_UN);
+      close(fd);
+      return fail(JITC_EIO, "jitc_register: mmap " + g.img_path + ": " + strerror(errno));
+    }
     cudaError_t e = cudaHostRegister(p, g.img_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+    flock(fd, LOCK_UN);
+    close(fd);
     if (e != cudaSuccess) {
       munmap(p, g.img_bytes);
       return fail(JITC_ENOMEM, std::string("jitc_register: cudaHostRegister: ") + cudaGetErrorString(e));

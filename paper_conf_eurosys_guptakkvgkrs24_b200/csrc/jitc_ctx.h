@@ -9,6 +9,7 @@
 #include <nccl.h>
 #include <stdio.h>
 #include <string.h>
+#include <sys/file.h>
 #include <sys/mman.h>
 #include <sys/stat.h>
 #include <sys/types.h>
