@@ -203,9 +203,12 @@ def run_jitc(args):
         if rank not in g.members:
             ctx.declare_group(g.group, g.policy, g.members)
     if world > 1:
-        uid = [J.get_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0)
-        ctx.comm_init(uid[0], world, rank)
+        if args.transport == "nccl":
+            uid = [J.get_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+            ctx.comm_init(uid[0], world, rank)
+        else:   # intra-node CUDA IPC transport (fresh directory per communicator)
+            ctx.comm_init_ipc(f"{shm}-comm", world, rank)
     torch.cuda.synchronize()
     setup_s = time.perf_counter() - t_setup
 
@@ -311,6 +314,7 @@ def run_jitc(args):
             "data": "synthetic training state (O9 integer generator; bf16 params, fp32 master/m/v, bf16 grads)",
             "config": {"workload": w.name, "image_bytes": L_total, "tensors": sum(len(g.tensors) for g in w.groups_of(rank)),
                        "writers_k": world, "restore_mode": "HOST", "image": "shared /dev/shm",
+                       "transport": args.transport if world > 1 else None,
                        "zero_copy": bool(args.zero_copy), "chunk_bytes": 1 << 20,
                        "staging_mib": args.staging, "slot_mib": args.slot,
                        "l2": f"state {L_total / 1e9:.1f} GB >> 126 MB L2; no flush needed", "setup_s": round(setup_s, 1)},
@@ -344,6 +348,7 @@ def run_jitc(args):
         dist.barrier()
     if rank == 0 and not args.image_dir:
         shutil.rmtree(shm, ignore_errors=True)
+        shutil.rmtree(f"{shm}-comm", ignore_errors=True)
 
 
 def main():
@@ -359,6 +364,8 @@ def main():
     ap.add_argument("--image-dir", default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
+    ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],
+                    help="N > 1 communicator: intra-node CUDA IPC (default; tested on B200 with real processes) or NCCL")
     ap.add_argument("--ref-sample", type=int, default=1024, help="MiB per reference step")
     args = ap.parse_args()
     if args.warmup < 3:

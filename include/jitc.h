@@ -186,6 +186,17 @@ jitc_status jitc_comm_init(jitc_ctx* ctx, const void* id128, int32_t nranks, int
  * comms; Table 7 shows this dominates recovery). */
 jitc_status jitc_comm_shrink(jitc_ctx* ctx, const int32_t* failed, int32_t n_failed);
 jitc_status jitc_comm_destroy(jitc_ctx* ctx);
+/* Intra-node IPC transport instead of NCCL, for ranks of ONE box.  The ranks
+ * share a control block in `comm_dir/ctl` (a fresh directory per
+ * communicator, like a unique id) and map each other's staging buffers with
+ * CUDA IPC.  Exchange, barrier and restore then need no NCCL: progress
+ * counters are written by the GPU in stream order (cuStreamWriteValue64 into
+ * the mapped control block) and polled by the peers, and K3 reads each
+ * peer's block directly from the peer's staging (NVLink peer loads), fusing
+ * the slice exchange into the unpack+verify kernel.  jitc_comm_shrink drops
+ * ranks; every other call behaves as with NCCL. */
+jitc_status jitc_comm_init_ipc(jitc_ctx* ctx, const char* comm_dir, int32_t nranks, int32_t comm_rank,
+                               const int32_t* job_ranks);
 
 /* ---- on failure: capture --------------------------------------------------- */
 /* A3 = K1: JF64 chunk digests of every registered byte of `group` (or all
@@ -278,7 +289,7 @@ jitc_status jitc_shard_range(uint64_t n_c, uint32_t k, uint32_t s, uint64_t* c0,
 /* The round schedule jitc_restore executes for `group` on comm rank
  * `comm_rank` of an n-rank communicator whose comm rank i is job rank
  * comm_job_ranks[i], given the staging geometry.  Output: a 24-B header
- * ('JITP', n_ops, round_bytes, slots) followed by n_ops 48-B operations
+ * ('JITP', n_ops, round_bytes, slots, n_rounds) followed by n_ops 48-B operations
  * {round, kind (1 H2D, 2 ALLGATHER, 3 PACK, 4 SEND, 5 RECV, 6 UNPACK,
  * 7 DIGEST_SEND, 8 DIGEST_RECV), slot, peer, image range [a, b), staging
  * offset, bytes}.  Only the group's members get operations

@@ -118,6 +118,7 @@ void jitc_destroy(jitc_ctx* c) {
   if (c->s_comp) cudaStreamSynchronize(c->s_comp);
   if (c->s_copy) cudaStreamSynchronize(c->s_copy);
   if (c->comm) ncclCommDestroy(c->comm);
+  ipc_destroy(c);
   for (auto& kv : c->groups) free_group(kv.second);
   for (int i = 0; i < jitc_ctx::kSlots; ++i) {
     if (c->ev_ready[i]) cudaEventDestroy(c->ev_ready[i]);
@@ -341,7 +342,7 @@ jitc_status jitc_comm_init(jitc_ctx* c, const void* id128, int32_t nranks, int32
 }
 
 jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_failed) {
-  if (!c || !c->comm) return fail(JITC_ESTATE, "jitc_comm_shrink: no communicator");
+  if (!c || !has_comm(c)) return fail(JITC_ESTATE, "jitc_comm_shrink: no communicator");
   if (n_failed < 0 || (n_failed && !failed)) return fail(JITC_EINVAL, "jitc_comm_shrink: bad list");
   CU(cudaSetDevice(c->device));
   std::vector<int> excl;
@@ -352,10 +353,22 @@ jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_faile
     excl.push_back(r);
   }
   std::sort(excl.begin(), excl.end());
-  ncclComm_t nc = nullptr;
-  NC(ncclCommShrink(c->comm, excl.data(), (int)excl.size(), &nc, nullptr, NCCL_SHRINK_ABORT));
-  ncclCommAbort(c->comm);
-  c->comm = nc;
+  if (c->ipc) {  // the IPC transport has nothing hung to abort: drop the ranks
+    std::vector<int> slot;
+    std::vector<uint8_t*> ps;
+    for (int i = 0; i < c->comm_n; ++i)
+      if (!std::binary_search(excl.begin(), excl.end(), i)) {
+        slot.push_back(c->ipc->slot[i]);
+        ps.push_back(c->ipc->peer_staging[i]);
+      }
+    c->ipc->slot = slot;
+    c->ipc->peer_staging = ps;
+  } else {
+    ncclComm_t nc = nullptr;
+    NC(ncclCommShrink(c->comm, excl.data(), (int)excl.size(), &nc, nullptr, NCCL_SHRINK_ABORT));
+    ncclCommAbort(c->comm);
+    c->comm = nc;
+  }
   std::vector<int32_t> job;
   for (int i = 0; i < c->comm_n; ++i)
     if (!std::binary_search(excl.begin(), excl.end(), i)) job.push_back(c->comm_job[i]);
@@ -369,6 +382,7 @@ jitc_status jitc_comm_destroy(jitc_ctx* c) {
   if (!c) return fail(JITC_EINVAL, "jitc_comm_destroy: null ctx");
   if (c->comm) ncclCommDestroy(c->comm);
   c->comm = nullptr;
+  ipc_destroy(c);
   c->comm_n = 0;
   c->comm_rank = -1;
   c->comm_job.clear();
@@ -422,6 +436,7 @@ jitc_status jitc_fingerprint(jitc_ctx* c, uint32_t group, void* blob, size_t cap
 // ------------------------------------------------------------ record exchange (C1)
 jitc_status jitc_exchange_records(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len) {
   if (!c || !mine || !all_len || len < sizeof(BlobHdr)) return fail(JITC_EINVAL, "jitc_exchange_records: bad argument");
+  if (c->ipc) return ipc_exchange(c, mine, len, all, cap, all_len);
   if (!c->comm) {
     *all_len = len;
     if (cap == 0) return JITC_OK;

@@ -71,6 +71,36 @@ struct GroupState {
 
 typedef CUresult (*PFN_writeValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 
+// ------------------------------------------------------------- IPC transport
+// Intra-node alternative to NCCL (jitc_ipc.cc): ranks share a control block
+// in a /dev/shm file and map each other's staging buffers with CUDA IPC.
+// Progress counters are written by the GPU in stream order
+// (cuStreamWriteValue64 into the mapped control block) and polled by the
+// peers' host threads; K3 reads a peer's block straight from its staging
+// (peer memory over NVLink), so the exchange is fused into the unpack.
+constexpr int kIpcMaxRanks = 64;
+constexpr int kIpcMaxGroups = 64;
+struct IpcCtl {
+  uint64_t arrive[kIpcMaxRanks];                  // barrier generations
+  uint64_t posted[kIpcMaxRanks][kIpcMaxGroups];   // rounds whose outgoing block is ready
+  uint64_t consumed[kIpcMaxRanks][kIpcMaxGroups]; // rounds whose incoming blocks were read
+  cudaIpcMemHandle_t staging[kIpcMaxRanks];
+  uint64_t staging_off[kIpcMaxRanks];
+  uint64_t published[kIpcMaxRanks];
+};
+struct IpcComm {
+  std::string dir;
+  IpcCtl* ctl = nullptr;      // host mapping of dir/ctl
+  uint8_t* ctl_dev = nullptr; // device alias (cudaHostRegister mapped)
+  size_t ctl_bytes = 0;
+  std::vector<int> slot;               // comm rank -> index into the IpcCtl arrays (stable across shrink)
+  std::vector<uint8_t*> peer_staging;  // by comm rank (own entry = ctx staging)
+  std::vector<void*> opened;
+  uint64_t barrier_gen = 0, exchange_gen = 0;
+  std::map<uint32_t, uint64_t> rounds;      // cumulative restore rounds per group slot
+  std::map<uint32_t, uint64_t> digest_gen;  // PEER digest hand-offs per group slot
+};
+
 }  // namespace jitc
 
 using namespace jitc;
@@ -103,6 +133,7 @@ struct jitc_ctx {
   ncclComm_t comm = nullptr;
   int comm_n = 0, comm_rank = -1;
   std::vector<int32_t> comm_job;  // comm rank -> job rank
+  std::unique_ptr<IpcComm> ipc;   // IPC transport (instead of `comm`)
   uint64_t* d_small = nullptr;    // 64 B device scratch for size exchange / barrier
   uint32_t* d_work = nullptr;     // K1/K2/K3 batch counters (self-resetting)
   uint64_t* h_small = nullptr;    // pinned
@@ -305,7 +336,20 @@ inline bool read_file(const std::string& path, std::vector<uint8_t>* out) {
   return ok;
 }
 
+}  // namespace jitc
+namespace jitc {
+// IPC transport (jitc_ipc.cc)
+jitc_status ipc_barrier(jitc_ctx* c);
+jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len);
+jitc_status ipc_post(jitc_ctx* c, uint64_t* counter, uint64_t value, cudaStream_t s);
+jitc_status ipc_wait(const uint64_t* counter, uint64_t value, const char* what);
+void ipc_destroy(jitc_ctx* c);
+uint32_t group_slot(const jitc_ctx* c, uint32_t group);
+
+inline bool has_comm(const jitc_ctx* c) { return c->comm || c->ipc; }
+
 inline jitc_status barrier(jitc_ctx* c) {
+  if (c->ipc) return ipc_barrier(c);
   if (!c->comm) return JITC_OK;
   NC(ncclAllReduce(c->d_small, c->d_small + 1, 1, ncclUint64, ncclSum, c->comm, c->s_comp));
   CU(cudaStreamSynchronize(c->s_comp));

@@ -247,7 +247,7 @@ struct PlanHdr {     // 24 B
   uint32_t n_ops;
   uint64_t round_bytes;
   uint32_t slots;
-  uint32_t pad;
+  uint32_t n_rounds;   // rounds every participant executes (some may carry no operation for this rank)
 };
 #pragma pack(pop)
 static_assert(sizeof(PlanOp) == 48, "plan op");
@@ -261,7 +261,7 @@ struct PlanInput {
   uint64_t staging_bytes = 0, slot_bytes = 0;
 };
 bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
-                        std::string* why);
+                        std::string* why, uint32_t* n_rounds = nullptr);
 uint64_t manifest_trailer(const uint8_t* p, size_t n);
 
 // thread-local error text

@@ -1,0 +1,198 @@
+// Intra-node IPC transport: the library communicator without NCCL.
+//
+// The ranks of one box share a control block (IpcCtl) in a /dev/shm file and
+// map each other's staging buffers through CUDA IPC.  Every signal is a
+// monotonically increasing counter:
+//   posted[r][g]   -- rank r's outgoing block of its restore round is ready,
+//   consumed[r][g] -- rank r has finished reading every block of a round,
+//   arrive[r]      -- barrier generation,
+// written by the GPU in stream order (cuStreamWriteValue64 into the
+// cudaHostRegister-mapped block, after the kernels / copies that produce or
+// consume the data) or by the host (barriers), and polled by the peers' host
+// threads before they enqueue dependent work.  A receiver's K3 reads the
+// sender's block straight out of the sender's staging buffer -- NVLink peer
+// loads on a multi-GPU node -- so the exchange and the unpack+verify are one
+// kernel.  The communicator's directory must be fresh for every communicator
+// (it plays the role of an NCCL unique id).
+#include <sched.h>
+
+#include "jitc_ctx.h"
+
+using namespace jitc;
+
+namespace {
+
+typedef CUresult (*PFN_getAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr);
+
+PFN_getAddressRange range_fn() {
+  static PFN_getAddressRange fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_getAddressRange)p;
+  }
+  return fn;
+}
+
+inline uint64_t load_acq(const uint64_t* p) { return __atomic_load_n(p, __ATOMIC_ACQUIRE); }
+inline void store_rel(uint64_t* p, uint64_t v) { __atomic_store_n(p, v, __ATOMIC_RELEASE); }
+
+constexpr double kIpcTimeoutMs = 600000.0;
+
+}  // namespace
+
+namespace jitc {
+
+uint32_t group_slot(const jitc_ctx* c, uint32_t group) {
+  uint32_t i = 0;
+  for (auto& kv : c->groups) {
+    if (kv.first == group) return i;
+    ++i;
+  }
+  return i;
+}
+
+jitc_status ipc_wait(const uint64_t* counter, uint64_t value, const char* what) {
+  const double t0 = now_ms();
+  uint32_t spins = 0;
+  while (load_acq(counter) < value) {
+    if (++spins > 1000) sched_yield();
+    if ((spins & 0xFFFF) == 0 && now_ms() - t0 > kIpcTimeoutMs)
+      return fail(JITC_ESTATE, std::string("IPC transport: timed out waiting for ") + what);
+  }
+  return JITC_OK;
+}
+
+jitc_status ipc_post(jitc_ctx* c, uint64_t* counter, uint64_t value, cudaStream_t s) {
+  uint64_t* dev = reinterpret_cast<uint64_t*>(c->ipc->ctl_dev + ((uint8_t*)counter - (uint8_t*)c->ipc->ctl));
+  if (c->write_value64 && c->write_value64((CUstream)s, (CUdeviceptr)dev, value, 0) == CUDA_SUCCESS) return JITC_OK;
+  CU(launch_phase_write(dev, value, s));
+  return JITC_OK;
+}
+
+jitc_status ipc_barrier(jitc_ctx* c) {
+  IpcComm& ic = *c->ipc;
+  const uint64_t gen = ++ic.barrier_gen;
+  store_rel(&ic.ctl->arrive[ic.slot[c->comm_rank]], gen);
+  for (int q = 0; q < c->comm_n; ++q) {
+    jitc_status st = ipc_wait(&ic.ctl->arrive[ic.slot[q]], gen, "a barrier");
+    if (st) return st;
+  }
+  return JITC_OK;
+}
+
+jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len) {
+  IpcComm& ic = *c->ipc;
+  // the two-call size query is collective too: both calls run the protocol
+  const uint64_t gen = ++ic.exchange_gen;
+  std::string me = ic.dir + "/blob." + std::to_string(gen) + "." + std::to_string(ic.slot[c->comm_rank]);
+  if (!write_file_atomic(me, static_cast<const uint8_t*>(mine), len))
+    return fail(JITC_EIO, "jitc_exchange_records: writing " + me);
+  jitc_status st = ipc_barrier(c);
+  if (st) return st;
+  std::vector<uint8_t> out;
+  for (int q = 0; q < c->comm_n; ++q) {
+    std::vector<uint8_t> b;
+    std::string p = ic.dir + "/blob." + std::to_string(gen) + "." + std::to_string(ic.slot[q]);
+    if (!read_file(p, &b)) return fail(JITC_EIO, "jitc_exchange_records: reading " + p);
+    out.insert(out.end(), b.begin(), b.end());
+  }
+  st = ipc_barrier(c);  // every rank has read every blob
+  if (st) return st;
+  unlink(me.c_str());
+  *all_len = out.size();
+  if (cap == 0) return JITC_OK;
+  if (cap < out.size() || !all) return fail(JITC_EINVAL, "jitc_exchange_records: buffer too small");
+  memcpy(all, out.data(), out.size());
+  return JITC_OK;
+}
+
+void ipc_destroy(jitc_ctx* c) {
+  if (!c->ipc) return;
+  IpcComm& ic = *c->ipc;
+  for (void* p : ic.opened) cudaIpcCloseMemHandle(p);
+  if (ic.ctl) {
+    cudaHostUnregister(ic.ctl);
+    munmap(ic.ctl, ic.ctl_bytes);
+  }
+  c->ipc.reset();
+}
+
+}  // namespace jitc
+
+extern "C" jitc_status jitc_comm_init_ipc(jitc_ctx* c, const char* comm_dir, int32_t nranks, int32_t comm_rank,
+                                          const int32_t* job_ranks) {
+  if (!c || !comm_dir || nranks <= 0 || nranks > kIpcMaxRanks || comm_rank < 0 || comm_rank >= nranks)
+    return fail(JITC_EINVAL, "jitc_comm_init_ipc: bad argument");
+  if (c->groups.size() > (size_t)kIpcMaxGroups) return fail(JITC_EINVAL, "jitc_comm_init_ipc: too many groups");
+  CU(cudaSetDevice(c->device));
+  if (c->comm) {
+    ncclCommDestroy(c->comm);
+    c->comm = nullptr;
+  }
+  ipc_destroy(c);
+  PFN_getAddressRange range = range_fn();
+  if (!range) return fail(JITC_ECUDA, "jitc_comm_init_ipc: cuMemGetAddressRange unavailable");
+  std::unique_ptr<IpcComm> ic(new IpcComm());
+  ic->dir = comm_dir;
+  mkdir(ic->dir.c_str(), 0700);
+  std::string path = ic->dir + "/ctl";
+  ic->ctl_bytes = align_up(sizeof(IpcCtl), 4096);
+  int fd = open(path.c_str(), O_RDWR | O_CREAT, 0600);
+  if (fd < 0) return fail(JITC_EIO, "jitc_comm_init_ipc: open " + path + ": " + strerror(errno));
+  flock(fd, LOCK_EX);
+  struct stat sb;
+  if (fstat(fd, &sb) == 0 && (uint64_t)sb.st_size < ic->ctl_bytes && ftruncate(fd, (off_t)ic->ctl_bytes) != 0) {
+    flock(fd, LOCK_UN);
+    close(fd);
+    return fail(JITC_EIO, "jitc_comm_init_ipc: sizing " + path);
+  }
+  void* p = mmap(nullptr, ic->ctl_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  cudaError_t e = p == MAP_FAILED ? cudaErrorMemoryAllocation
+                                  : cudaHostRegister(p, ic->ctl_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+  flock(fd, LOCK_UN);
+  close(fd);
+  if (p == MAP_FAILED) return fail(JITC_EIO, "jitc_comm_init_ipc: mmap " + path);
+  if (e != cudaSuccess) {
+    munmap(p, ic->ctl_bytes);
+    return fail(JITC_ECUDA, std::string("jitc_comm_init_ipc: cudaHostRegister: ") + cudaGetErrorString(e));
+  }
+  ic->ctl = static_cast<IpcCtl*>(p);
+  CU(cudaHostGetDevicePointer((void**)&ic->ctl_dev, p, 0));
+  // publish this rank's staging
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (range(&base, &size, (CUdeviceptr)c->staging) != CUDA_SUCCESS)
+    return fail(JITC_ECUDA, "jitc_comm_init_ipc: staging is not device memory");
+  cudaIpcMemHandle_t h;
+  e = cudaIpcGetMemHandle(&h, (void*)base);
+  if (e != cudaSuccess)
+    return fail(JITC_ECUDA, std::string("jitc_comm_init_ipc: cudaIpcGetMemHandle(staging): ") + cudaGetErrorString(e));
+  ic->ctl->staging[comm_rank] = h;
+  ic->ctl->staging_off[comm_rank] = (uint64_t)c->staging - (uint64_t)base;
+  store_rel(&ic->ctl->published[comm_rank], 1);
+  ic->slot.resize(nranks);
+  for (int i = 0; i < nranks; ++i) ic->slot[i] = i;
+  ic->peer_staging.assign(nranks, nullptr);
+  ic->peer_staging[comm_rank] = c->staging;
+  c->comm_n = nranks;
+  c->comm_rank = comm_rank;
+  c->comm_job.resize(nranks);
+  for (int i = 0; i < nranks; ++i) c->comm_job[i] = job_ranks ? job_ranks[i] : i;
+  if (c->comm_job[comm_rank] != c->cfg.rank) return fail(JITC_EINVAL, "jitc_comm_init_ipc: job_ranks[comm_rank] != cfg.rank");
+  for (int q = 0; q < nranks; ++q) {
+    if (q == comm_rank) continue;
+    jitc_status st = ipc_wait(&ic->ctl->published[q], 1, "a peer to publish its staging");
+    if (st) return st;
+    void* m = nullptr;
+    e = cudaIpcOpenMemHandle(&m, ic->ctl->staging[q], cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess)
+      return fail(JITC_ECUDA, std::string("jitc_comm_init_ipc: cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+    ic->opened.push_back(m);
+    ic->peer_staging[q] = static_cast<uint8_t*>(m) + ic->ctl->staging_off[q];
+  }
+  c->ipc = std::move(ic);
+  return ipc_barrier(c);
+}

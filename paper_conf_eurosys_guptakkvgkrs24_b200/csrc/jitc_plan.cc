@@ -30,10 +30,13 @@ static void o5_bytes(uint64_t n_c, uint64_t k, uint64_t s, uint64_t C, uint64_t 
 }
 
 bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
-                        std::string* why) {
+                        std::string* why, uint32_t* n_rounds) {
   ops->clear();
   *round_bytes = 0;
   *slots = 0;
+  uint32_t dummy_rounds;
+  if (!n_rounds) n_rounds = &dummy_rounds;
+  *n_rounds = 0;
   const uint64_t C = in.chunk_bytes, L = in.image_bytes, n_c = in.n_c;
   if (C == 0 || in.n <= 0 || in.me < 0 || in.me >= in.n) {
     *why = "bad plan input";
@@ -63,6 +66,7 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
       maxlen = std::max(maxlen, q1[r] - q0[r]);
     }
     const uint64_t J = (maxlen + R - 1) / R;
+    *n_rounds = (uint32_t)J;
     for (uint64_t j = 0; j < J; ++j) {
       const uint32_t sl = (uint32_t)(j % S);
       const uint64_t base = sl * n * R;
@@ -121,14 +125,16 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
     maxlen = std::max(maxlen, q1[s] - q0[s]);
   }
   const uint64_t J = (maxlen + R - 1) / R;
+  *n_rounds = (uint32_t)J;
   for (uint64_t j = 0; j < J; ++j) {
     const uint32_t sl = (uint32_t)(j % S);
-    const uint64_t base = sl * k * R;
+    const uint64_t base = sl * k * R;   // block s of a round sits at base + s*R on every rank
     if (my_s >= 0) {
       uint64_t a = q0[my_s] + j * R, b = std::min(q1[my_s], a + R);
       if (b <= a) continue;
-      ops->push_back(PlanOp{(uint32_t)j, kOpPack, (uint8_t)sl, 0, in.me, 0, a, b, base, b - a});
-      for (int32_t d : in.dests) ops->push_back(PlanOp{(uint32_t)j, kOpSend, (uint8_t)sl, 0, d, 0, a, b, base, b - a});
+      const uint64_t off = base + (uint64_t)my_s * R;
+      ops->push_back(PlanOp{(uint32_t)j, kOpPack, (uint8_t)sl, 0, in.me, 0, a, b, off, b - a});
+      for (int32_t d : in.dests) ops->push_back(PlanOp{(uint32_t)j, kOpSend, (uint8_t)sl, 0, d, 0, a, b, off, b - a});
     } else {
       for (uint64_t s = 0; s < k; ++s) {
         uint64_t a = q0[s] + j * R, b = std::min(q1[s], a + R);
@@ -193,8 +199,8 @@ extern "C" jitc_status jitc_restore_plan(const void* selection, size_t sel_len, 
   }
   std::vector<PlanOp> ops;
   uint64_t R = 0;
-  uint32_t S = 0;
-  if (!build_restore_plan(in, &ops, &R, &S, &why)) {
+  uint32_t S = 0, J = 0;
+  if (!build_restore_plan(in, &ops, &R, &S, &why, &J)) {
     set_error("jitc_restore_plan: " + why);
     return JITC_EINVAL;
   }
@@ -203,6 +209,7 @@ extern "C" jitc_status jitc_restore_plan(const void* selection, size_t sel_len, 
   h.n_ops = (uint32_t)ops.size();
   h.round_bytes = R;
   h.slots = S;
+  h.n_rounds = J;
   *len = sizeof h + ops.size() * sizeof(PlanOp);
   if (cap == 0) return JITC_OK;
   if (cap < *len || !plan) {

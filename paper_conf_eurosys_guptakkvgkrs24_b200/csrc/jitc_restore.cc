@@ -71,24 +71,37 @@ jitc_status jitc::compare_digests(jitc_ctx* c, GroupState& g, const std::vector<
 }
 
 // Executes a restore plan (jitc_plan.cc) round by round: H2D on the copy
-// stream; K2 packs, NCCL send/recv or all-gather and K3 unpacks on the
-// compute stream; slot reuse ordered by the ready/free events.
-static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<PlanOp>& ops, uint32_t S,
-                                jitc_stats* stats) {
+// stream; K2 packs, the exchange and K3 unpacks on the compute stream; slot
+// reuse ordered by the ready/free events.  The exchange is NCCL (send/recv or
+// in-place all-gather) or, with the IPC transport, nothing at all: K3 reads a
+// peer's block straight from the peer's staging once the peer has posted it,
+// and every rank posts / consumes every round (counters in shared memory)
+// so that senders know when a slot may be refilled.
+static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<PlanOp>& ops, uint32_t S, uint32_t J,
+                                const std::vector<int>& readers, jitc_stats* stats) {
   if (S > (uint32_t)jitc_ctx::kSlots) return fail(JITC_EINVAL, "execute_plan: too many slots");
+  IpcComm* ic = c->ipc.get();
+  const uint32_t gs = ic ? group_slot(c, g.id) : 0;
+  const uint64_t base_round = ic ? ic->rounds[gs] : 0;
+  const int my_slot = ic ? ic->slot[c->comm_rank] : 0;
   bool used[jitc_ctx::kSlots] = {false};
   size_t i = 0;
   uint32_t rounds = 0;
-  while (i < ops.size()) {
-    if (ops[i].kind == kOpDigestSend || ops[i].kind == kOpDigestRecv) {
-      ++i;
-      continue;
-    }
-    const uint32_t j = ops[i].round;
+  for (uint32_t j = 0; j < J; ++j) {
+    while (i < ops.size() && (ops[i].kind == kOpDigestSend || ops[i].kind == kOpDigestRecv)) ++i;
     size_t e = i;
     while (e < ops.size() && ops[e].round == j && ops[e].kind != kOpDigestSend && ops[e].kind != kOpDigestRecv) ++e;
-    const uint32_t sl = ops[i].slot;
-    ++rounds;
+    const uint32_t sl = j % (S ? S : 1);
+    const uint64_t seq = base_round + j + 1;  // IPC: this round's counter value
+    bool writes_slot = false;
+    for (size_t q = i; q < e; ++q) writes_slot |= ops[q].kind == kOpH2D || ops[q].kind == kOpPack;
+    if (e > i) ++rounds;
+    // 0. IPC: the readers of my slot must have consumed the round that used it last
+    if (ic && writes_slot && j >= S)
+      for (int r : readers) {
+        jitc_status st = ipc_wait(&ic->ctl->consumed[ic->slot[r]][gs], seq - S, "a peer to consume a round");
+        if (st) return st;
+      }
     // 1. host -> device on the copy stream
     bool any_h2d = false;
     for (size_t q = i; q < e; ++q) {
@@ -112,27 +125,40 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
       jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, c->staging + op.off, op.a), g.d_dig2, op.b - op.a);
       if (st) return st;
     }
-    // 3. NCCL: point-to-point (PEER) and all-gather (HOST, n > 1)
-    bool p2p = false;
-    for (size_t q = i; q < e; ++q) p2p |= ops[q].kind == kOpSend || ops[q].kind == kOpRecv;
-    if (p2p) {
-      NC(ncclGroupStart());
+    // 3. the exchange
+    if (ic) {
+      jitc_status st = ipc_post(c, &ic->ctl->posted[my_slot][gs], seq, c->s_comp);  // my block is ready
+      if (st) return st;
       for (size_t q = i; q < e; ++q) {
         const PlanOp& op = ops[q];
-        if (op.kind == kOpSend) NC(ncclSend(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
-        if (op.kind == kOpRecv) NC(ncclRecv(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
-        if (stats) stats->p2p_bytes += op.bytes;
+        if (op.kind != kOpUnpack || op.peer == c->comm_rank) continue;
+        st = ipc_wait(&ic->ctl->posted[ic->slot[op.peer]][gs], seq, "a peer to post a round");
+        if (st) return st;
+        if (stats) stats->p2p_bytes += op.b - op.a;
       }
-      NC(ncclGroupEnd());
+    } else {
+      bool p2p = false;
+      for (size_t q = i; q < e; ++q) p2p |= ops[q].kind == kOpSend || ops[q].kind == kOpRecv;
+      if (p2p) {
+        NC(ncclGroupStart());
+        for (size_t q = i; q < e; ++q) {
+          const PlanOp& op = ops[q];
+          if (op.kind == kOpSend) NC(ncclSend(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+          if (op.kind == kOpRecv) NC(ncclRecv(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+          if (stats) stats->p2p_bytes += op.bytes;
+        }
+        NC(ncclGroupEnd());
+      }
+      for (size_t q = i; q < e; ++q) {
+        const PlanOp& op = ops[q];
+        if (op.kind != kOpAllGather) continue;
+        uint8_t* base = c->staging + op.off;
+        NC(ncclAllGather(base + (uint64_t)c->comm_rank * op.bytes, base, op.bytes, ncclUint8, c->comm, c->s_comp));
+        if (stats) stats->p2p_bytes += (uint64_t)(c->comm_n - 1) * op.bytes;
+      }
     }
-    for (size_t q = i; q < e; ++q) {
-      const PlanOp& op = ops[q];
-      if (op.kind != kOpAllGather) continue;
-      uint8_t* base = c->staging + op.off;
-      NC(ncclAllGather(base + (uint64_t)c->comm_rank * op.bytes, base, op.bytes, ncclUint8, c->comm, c->s_comp));
-      if (stats) stats->p2p_bytes += (uint64_t)(c->comm_n - 1) * op.bytes;
-    }
-    // 4. K3 unpack + verify of every block of the round (<= kMaxRanges per launch)
+    // 4. K3 unpack + verify of every block of the round (<= kMaxRanges per launch);
+    //    with IPC a peer's block is read in place from the peer's staging
     LaunchRanges lr{};
     uint64_t bytes = 0;
     for (size_t q = i; q < e; ++q) {
@@ -140,7 +166,8 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
       if (op.kind != kOpUnpack) continue;
       uint32_t lo, hi;
       seg_span(g, op.a, op.b, &lo, &hi);
-      add_range(lr, lo, hi, c->staging + op.off, op.a);
+      const uint8_t* src = (ic && op.peer != c->comm_rank) ? ic->peer_staging[op.peer] + op.off : c->staging + op.off;
+      add_range(lr, lo, hi, src, op.a);
       bytes += op.b - op.a;
       if (lr.n == kMaxRanges) {
         jitc_status st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
@@ -153,18 +180,32 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
       jitc_status st = run_segments(c, g, kUnpack, lr, g.d_dig2, bytes);
       if (st) return st;
     }
-    CU(cudaEventRecord(c->ev_free[sl], c->s_comp));
-    used[sl] = true;
+    if (ic) {
+      jitc_status st = ipc_post(c, &ic->ctl->consumed[my_slot][gs], seq, c->s_comp);  // done reading this round
+      if (st) return st;
+    }
+    if (e > i) {
+      CU(cudaEventRecord(c->ev_free[sl], c->s_comp));
+      used[sl] = true;
+    }
     i = e;
+  }
+  if (ic) {
+    // my staging may be reused as soon as this call returns: wait for its readers
+    for (int r : readers) {
+      jitc_status st = ipc_wait(&ic->ctl->consumed[ic->slot[r]][gs], base_round + J, "a peer to finish reading");
+      if (st) return st;
+    }
+    ic->rounds[gs] = base_round + J;
   }
   if (stats) stats->rounds += rounds;
   return JITC_OK;
 }
 
-static jitc_status make_plan(jitc_ctx* c, const PlanInput& in, std::vector<PlanOp>* ops, uint32_t* S) {
+static jitc_status make_plan(jitc_ctx* c, const PlanInput& in, std::vector<PlanOp>* ops, uint32_t* S, uint32_t* J) {
   uint64_t R;
   std::string why;
-  if (!build_restore_plan(in, ops, &R, S, &why)) return fail(JITC_ENOMEM, "jitc_restore: " + why);
+  if (!build_restore_plan(in, ops, &R, S, &why, J)) return fail(JITC_ENOMEM, "jitc_restore: " + why);
   return JITC_OK;
 }
 
@@ -176,7 +217,7 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
   jitc_status st = load_manifest(c, g, &mv);
   if (st) return st;
   if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
-  const int n = c->comm ? c->comm_n : 1;
+  const int n = has_comm(c) ? c->comm_n : 1;
   if (n > 1 && !g.img_shm)
     return fail(JITC_EINVAL, "jitc_restore: HOST mode across ranks needs a shared image_dir (use PEER mode)");
   if (n == 1 && (c->cfg.flags & JITC_F_ZERO_COPY_H2D)) {
@@ -190,10 +231,10 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
     in.chunk_bytes = g.C;
     in.image_bytes = g.L;
     in.n = n;
-    in.me = c->comm ? c->comm_rank : 0;
+    in.me = has_comm(c) ? c->comm_rank : 0;
     in.staging_bytes = c->staging_bytes;
     in.slot_bytes = c->slot_bytes;
-    if (c->comm) {
+    if (has_comm(c)) {
       for (int32_t m : g.members) {
         int r = comm_rank_of(c, m);
         if (r >= 0) in.participants.push_back(r);
@@ -203,10 +244,14 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
       in.participants = {0};
     }
     std::vector<PlanOp> ops;
-    uint32_t S = 0;
-    st = make_plan(c, in, &ops, &S);
+    uint32_t S = 0, J = 0;
+    st = make_plan(c, in, &ops, &S, &J);
     if (st) return st;
-    st = execute_plan(c, g, ops, S, stats);
+    std::vector<int> readers;  // every other member reads my slice
+    for (int r : in.participants)
+      if (r != in.me) readers.push_back(r);
+    if (std::find(in.participants.begin(), in.participants.end(), in.me) == in.participants.end()) readers.clear();
+    st = execute_plan(c, g, ops, S, J, readers, stats);
     if (st) return st;
   }
   st = compare_digests(c, g, mv.d, stats);
@@ -222,7 +267,7 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
 // and send them over NVLink to every member that is not a writer; receivers
 // unpack+verify (K3) against the writers' digests (broadcast first).
 static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection& gs, jitc_stats* stats) {
-  if (!c->comm) return fail(JITC_ESTATE, "jitc_restore: PEER mode needs a communicator");
+  if (!has_comm(c)) return fail(JITC_ESTATE, "jitc_restore: PEER mode needs a communicator");
   if (gs.writers.empty()) return JITC_OK;  // dropped OPTIONAL group
   if (gs.layout_hash != g.layout_hash || gs.n_c != g.n_c || gs.image_bytes != g.L)
     return fail(JITC_ELAYOUT, "jitc_restore: selection layout differs from the registered one");
@@ -249,8 +294,8 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   const bool is_writer = my_s < (int)in.writers.size();
   const bool is_dst = std::find(in.dests.begin(), in.dests.end(), in.me) != in.dests.end();
   std::vector<PlanOp> ops;
-  uint32_t S = 0;
-  jitc_status st = make_plan(c, in, &ops, &S);
+  uint32_t S = 0, J = 0;
+  jitc_status st = make_plan(c, in, &ops, &S, &J);
   if (st) return st;
   if (!is_writer && !is_dst) return JITC_OK;
   // 1. the lowest writer sends the selected class's digests to every destination
@@ -261,7 +306,24 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
     CU(cudaMemcpyAsync(d_expect, g.fp.data(), g.n_c * 8, cudaMemcpyHostToDevice, c->s_comp));
   bool any = false;
   for (const PlanOp& op : ops) any |= op.kind == kOpDigestSend || op.kind == kOpDigestRecv;
-  if (any && g.n_c) {
+  if (c->ipc) {
+    // IPC: the lowest writer leaves the digests in a file of the communicator
+    // directory (per group and hand-off generation); receivers wait for it.
+    const uint32_t gsl = group_slot(c, g.id);
+    const uint64_t gen = ++c->ipc->digest_gen[gsl];
+    const std::string path = c->ipc->dir + "/dig." + std::to_string(gsl) + "." + std::to_string(gen);
+    if (is_writer && my_s == 0 && !write_file_atomic(path, reinterpret_cast<const uint8_t*>(g.fp.data()), 8 * g.n_c))
+      return fail(JITC_EIO, "jitc_restore: writing " + path);
+    if (is_dst) {
+      std::vector<uint8_t> b;
+      const double t0 = now_ms();
+      while (!read_file(path, &b) || b.size() != 8 * g.n_c) {
+        if (now_ms() - t0 > 600000.0) return fail(JITC_ESTATE, "jitc_restore: no digests from the writers");
+        usleep(200);
+      }
+      if (g.n_c) CU(cudaMemcpyAsync(d_expect, b.data(), g.n_c * 8, cudaMemcpyHostToDevice, c->s_comp));
+    }
+  } else if (any && g.n_c) {
     NC(ncclGroupStart());
     for (const PlanOp& op : ops) {
       if (op.kind == kOpDigestSend) NC(ncclSend(d_expect, g.n_c, ncclUint64, op.peer, c->comm, c->s_comp));
@@ -280,7 +342,9 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   }
   if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
   // 2. data rounds
-  st = execute_plan(c, g, ops, S, stats);
+  std::vector<int> readers;  // a writer's blocks are read by every destination
+  if (is_writer) readers = in.dests;
+  st = execute_plan(c, g, ops, S, J, readers, stats);
   if (st) return st;
   CU(cudaStreamSynchronize(c->s_comp));
   if (is_dst) {

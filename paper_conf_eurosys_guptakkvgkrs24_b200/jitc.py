@@ -90,6 +90,7 @@ def lib() -> ctypes.CDLL:
         "jitc_comm_init": ([vp, vp, i32, i32, P(i32)], i32),
         "jitc_comm_shrink": ([vp, P(i32), i32], i32),
         "jitc_comm_destroy": ([vp], i32),
+        "jitc_comm_init_ipc": ([vp, ctypes.c_char_p, i32, i32, P(i32)], i32),
         "jitc_fingerprint": ([vp, u32, vp, sz, P(sz)], i32),
         "jitc_exchange_records": ([vp, vp, sz, vp, sz, P(sz)], i32),
         "jitc_select_consistent_replica": ([vp, sz, P(i32), i32, vp, sz, P(sz)], i32),
@@ -129,7 +130,7 @@ def lib() -> ctypes.CDLL:
 
 EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version", "jitc_register",
             "jitc_declare_group", "jitc_mark", "jitc_phase", "jitc_get_unique_id", "jitc_comm_init",
-            "jitc_comm_shrink", "jitc_comm_destroy", "jitc_fingerprint", "jitc_exchange_records",
+            "jitc_comm_shrink", "jitc_comm_destroy", "jitc_comm_init_ipc", "jitc_fingerprint", "jitc_exchange_records",
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
@@ -227,12 +228,12 @@ def restore_plan(selection: bytes, group: int, mode: int, comm_job_ranks: Sequen
     buf = ctypes.create_string_buffer(n.value)
     _check(L.jitc_restore_plan(*args, buf, n.value, ctypes.byref(n)), "jitc_restore_plan")
     raw = buf.raw[:n.value]
-    magic, n_ops, R, S, _ = struct.unpack_from("<IIQII", raw, 0)
+    magic, n_ops, R, S, n_rounds = struct.unpack_from("<IIQII", raw, 0)
     ops = []
     for i in range(n_ops):
         rnd, kind, slot, _p, peer, _p2, a, b, off, nb = struct.unpack_from("<IBBHiIQQQQ", raw, 24 + 48 * i)
         ops.append(dict(round=rnd, kind=OP_NAMES[kind], slot=slot, peer=peer, a=a, b=b, off=off, bytes=nb))
-    return dict(round_bytes=R, slots=S, ops=ops)
+    return dict(round_bytes=R, slots=S, n_rounds=n_rounds, ops=ops)
 
 
 def get_unique_id() -> bytes:
@@ -328,6 +329,11 @@ class Context:
     def comm_init(self, uid: bytes, nranks: int, comm_rank: int, job_ranks: Optional[Sequence[int]] = None):
         jr = _i32arr(list(job_ranks)) if job_ranks is not None else None
         _check(self._L.jitc_comm_init(self._h, uid, nranks, comm_rank, jr), "jitc_comm_init")
+
+    def comm_init_ipc(self, comm_dir: str, nranks: int, comm_rank: int, job_ranks: Optional[Sequence[int]] = None):
+        """Intra-node communicator over CUDA IPC + shared memory (no NCCL)."""
+        jr = _i32arr(list(job_ranks)) if job_ranks is not None else None
+        _check(self._L.jitc_comm_init_ipc(self._h, comm_dir.encode(), nranks, comm_rank, jr), "jitc_comm_init_ipc")
 
     def comm_shrink(self, failed: Sequence[int]):
         _check(self._L.jitc_comm_shrink(self._h, _i32arr(list(failed)), len(failed)), "jitc_comm_shrink")
