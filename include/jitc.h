@@ -327,7 +327,13 @@ jitc_status jitc_stage_in(jitc_ctx* ctx, uint32_t group, const char* dir, jitc_s
  * and stops.  While the watchdog runs, other threads may call only
  * jitc_watch_event / jitc_watchdog_wait / jitc_watchdog_stop on the ctx. */
 typedef void (*jitc_hang_fn)(void* user, uint64_t tag, double waited_ms);
-enum { JITC_ON_HANG_NOTIFY = 0, JITC_ON_HANG_LOCAL_CAPTURE = 1 };
+/* JITC_ON_HANG_COLLECTIVE_CAPTURE (IPC transport): peers whose heartbeat (a
+ * thread started by jitc_comm_init_ipc refreshes it every 10 ms) is older
+ * than timeout_ms are dead; the survivors drop them (jitc_comm_shrink) and
+ * run fingerprint -> exchange -> select -> sharded capture -> commit among
+ * themselves on their watchdog threads -- the paper's whole user-level
+ * protocol with no Python and no scheduler. */
+enum { JITC_ON_HANG_NOTIFY = 0, JITC_ON_HANG_LOCAL_CAPTURE = 1, JITC_ON_HANG_COLLECTIVE_CAPTURE = 2 };
 jitc_status jitc_watch_event(jitc_ctx* ctx, void* event, uint64_t tag);
 jitc_status jitc_watchdog_start(jitc_ctx* ctx, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user);
 /* Blocks up to max_ms for the hang action to finish.  *fired = 1 if it did;
@@ -335,6 +341,8 @@ jitc_status jitc_watchdog_start(jitc_ctx* ctx, uint32_t timeout_ms, int32_t acti
 jitc_status jitc_watchdog_wait(jitc_ctx* ctx, uint32_t max_ms, int32_t* fired, uint64_t* tag, double* waited_ms,
                                double* action_ms, jitc_stats* action_stats);
 jitc_status jitc_watchdog_stop(jitc_ctx* ctx);
+/* Job ranks the collective action found dead (up to cap; *n = count). */
+jitc_status jitc_watchdog_failed(jitc_ctx* ctx, int32_t* ranks, int32_t cap, int32_t* n);
 
 /* ---- analytic model (NEXT-3; §5, eqs. 1-8) ------------------------ */
 enum { JITC_MODEL_PERIODIC_OPTIMAL = 0, JITC_MODEL_PERIODIC = 1, JITC_MODEL_USER_JIT = 2,

@@ -17,6 +17,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <atomic>
 #include <condition_variable>
 #include <mutex>
 #include <thread>
@@ -87,6 +88,7 @@ struct IpcCtl {
   cudaIpcMemHandle_t staging[kIpcMaxRanks];
   uint64_t staging_off[kIpcMaxRanks];
   uint64_t published[kIpcMaxRanks];
+  uint64_t heartbeat[kIpcMaxRanks];  // CLOCK_MONOTONIC microseconds, refreshed every 10 ms while alive
 };
 struct IpcComm {
   std::string dir;
@@ -99,6 +101,8 @@ struct IpcComm {
   uint64_t barrier_gen = 0, exchange_gen = 0;
   std::map<uint32_t, uint64_t> rounds;      // cumulative restore rounds per group slot
   std::map<uint32_t, uint64_t> digest_gen;  // PEER digest hand-offs per group slot
+  std::thread hb_thread;                    // heartbeat writer (failure localisation, NEXT-1)
+  std::atomic<bool> hb_run{false};
 };
 
 }  // namespace jitc
@@ -156,6 +160,7 @@ struct jitc_ctx {
   void* hang_user = nullptr;
   jitc_status action_status = JITC_OK;
   jitc_stats action_stats{};
+  std::vector<int32_t> fired_failed;  // job ranks the collective action found dead
   // counters
   jitc_kernel_counter kc[5]{};
   uint64_t launches_in_call = 0;
@@ -343,6 +348,8 @@ jitc_status ipc_barrier(jitc_ctx* c);
 jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len);
 jitc_status ipc_post(jitc_ctx* c, uint64_t* counter, uint64_t value, cudaStream_t s);
 jitc_status ipc_wait(const uint64_t* counter, uint64_t value, const char* what);
+// job ranks of the communicator whose heartbeat is older than stale_ms (dead processes)
+std::vector<int32_t> ipc_stale_ranks(jitc_ctx* c, double stale_ms);
 void ipc_destroy(jitc_ctx* c);
 uint32_t group_slot(const jitc_ctx* c, uint32_t group);
 

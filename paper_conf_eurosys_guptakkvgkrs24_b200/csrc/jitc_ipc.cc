@@ -109,9 +109,28 @@ jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, s
   return JITC_OK;
 }
 
+static uint64_t mono_us() {
+  return (uint64_t)std::chrono::duration_cast<std::chrono::microseconds>(
+             std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+std::vector<int32_t> ipc_stale_ranks(jitc_ctx* c, double stale_ms) {
+  std::vector<int32_t> out;
+  if (!c->ipc) return out;
+  const uint64_t now = mono_us();
+  for (int q = 0; q < c->comm_n; ++q) {
+    if (q == c->comm_rank) continue;
+    uint64_t hb = load_acq(&c->ipc->ctl->heartbeat[c->ipc->slot[q]]);
+    if (hb == 0 || now > hb + (uint64_t)(stale_ms * 1000.0)) out.push_back(c->comm_job[q]);
+  }
+  return out;
+}
+
 void ipc_destroy(jitc_ctx* c) {
   if (!c->ipc) return;
   IpcComm& ic = *c->ipc;
+  ic.hb_run = false;
+  if (ic.hb_thread.joinable()) ic.hb_thread.join();
   for (void* p : ic.opened) cudaIpcCloseMemHandle(p);
   if (ic.ctl) {
     cudaHostUnregister(ic.ctl);
@@ -193,6 +212,17 @@ extern "C" jitc_status jitc_comm_init_ipc(jitc_ctx* c, const char* comm_dir, int
     ic->opened.push_back(m);
     ic->peer_staging[q] = static_cast<uint8_t*>(m) + ic->ctl->staging_off[q];
   }
+  // heartbeat: lets the survivors of a hang tell a dead peer from a hung one
+  store_rel(&ic->ctl->heartbeat[comm_rank], mono_us());
+  ic->hb_run = true;
+  IpcCtl* ctl = ic->ctl;
+  IpcComm* icp = ic.get();
+  ic->hb_thread = std::thread([ctl, icp, comm_rank] {
+    while (icp->hb_run) {
+      store_rel(&ctl->heartbeat[comm_rank], mono_us());
+      std::this_thread::sleep_for(std::chrono::milliseconds(10));
+    }
+  });
   c->ipc = std::move(ic);
   return ipc_barrier(c);
 }

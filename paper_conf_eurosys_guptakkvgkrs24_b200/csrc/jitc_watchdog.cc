@@ -12,6 +12,51 @@ using namespace jitc;
 // watchdog thread itself -- here entirely in C++ (no Python callback, so the
 // GIL cannot block it) on the library's non-blocking streams.
 
+// The paper's user-level protocol run by the survivors themselves
+// (PAPER.md:105-116): peers whose heartbeat went stale are dead; drop them
+// from the communicator (ncclCommShrink(ABORT), which also aborts the hung
+// collective, or an IPC shrink), then fingerprint -> exchange -> select ->
+// sharded capture -> commit among the survivors, all on this thread.
+static jitc_status collective_capture(jitc_ctx* c, jitc_stats* st) {
+  std::vector<int32_t> failed;
+  if (c->ipc) {
+    failed = ipc_stale_ranks(c, c->timeout_ms);
+  } else if (!c->comm) {
+    return local_capture(c, st);
+  } else {
+    return fail(JITC_ESTATE, "collective capture needs failure localisation: use the IPC transport "
+                             "(heartbeats) or JITC_ON_HANG_NOTIFY and shrink from the harness");
+  }
+  jitc_status r = JITC_OK;
+  if (!failed.empty()) {
+    r = jitc_comm_shrink(c, failed.data(), (int32_t)failed.size());
+    if (r) return r;
+  }
+  c->fired_failed = failed;
+  size_t len = 0;
+  r = jitc_fingerprint(c, JITC_ALL_GROUPS, nullptr, 0, &len);
+  if (r) return r;
+  std::vector<uint8_t> blob(len);
+  r = jitc_fingerprint(c, JITC_ALL_GROUPS, blob.data(), blob.size(), &len);
+  if (r) return r;
+  size_t all_len = 0;
+  r = jitc_exchange_records(c, blob.data(), len, nullptr, 0, &all_len);
+  if (r) return r;
+  std::vector<uint8_t> all(all_len);
+  r = jitc_exchange_records(c, blob.data(), len, all.data(), all.size(), &all_len);
+  if (r) return r;
+  size_t sl = 0;
+  jitc_select_consistent_replica(all.data(), all_len, c->comm_job.data(), (int32_t)c->comm_job.size(), nullptr, 0,
+                                 &sl);
+  std::vector<uint8_t> sel(sl);
+  r = jitc_select_consistent_replica(all.data(), all_len, c->comm_job.data(), (int32_t)c->comm_job.size(),
+                                     sel.data(), sel.size(), &sl);
+  if (r) return r;
+  r = jitc_capture(c, sel.data(), sl, JITC_ALL_GROUPS, st);
+  if (r) return r;
+  return commit_impl(c, sel.data(), sl, true);
+}
+
 static void watchdog_loop(jitc_ctx* c) {
   cudaSetDevice(c->device);
   const double t0 = now_ms();
@@ -40,9 +85,9 @@ static void watchdog_loop(jitc_ctx* c) {
       c->detect_ms = now - t0;
       lk.unlock();
       double ta = now_ms();
-      if (c->action == JITC_ON_HANG_LOCAL_CAPTURE) {
+      if (c->action == JITC_ON_HANG_LOCAL_CAPTURE || c->action == JITC_ON_HANG_COLLECTIVE_CAPTURE) {
         jitc_stats st{};
-        jitc_status r = local_capture(c, &st);
+        jitc_status r = c->action == JITC_ON_HANG_LOCAL_CAPTURE ? local_capture(c, &st) : collective_capture(c, &st);
         lk.lock();
         c->action_status = r;
         c->action_stats = st;
@@ -79,7 +124,8 @@ jitc_status jitc_watch_event(jitc_ctx* c, void* event, uint64_t tag) {
 
 jitc_status jitc_watchdog_start(jitc_ctx* c, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user) {
   if (!c) return fail(JITC_EINVAL, "jitc_watchdog_start: null ctx");
-  if (action != JITC_ON_HANG_NOTIFY && action != JITC_ON_HANG_LOCAL_CAPTURE)
+  if (action != JITC_ON_HANG_NOTIFY && action != JITC_ON_HANG_LOCAL_CAPTURE &&
+      action != JITC_ON_HANG_COLLECTIVE_CAPTURE)
     return fail(JITC_EINVAL, "jitc_watchdog_start: bad action");
   stop_thread(c);  // a previous watchdog; the watch-list is kept
   std::lock_guard<std::mutex> lk(c->wmu);
@@ -109,6 +155,14 @@ jitc_status jitc_watchdog_wait(jitc_ctx* c, uint32_t max_ms, int32_t* fired, uin
   jitc_status st = c->action_done ? c->action_status : JITC_OK;
   if (st) set_error("jitc_watchdog_wait: the on-hang capture failed with status " + std::to_string(st));
   return st;
+}
+
+jitc_status jitc_watchdog_failed(jitc_ctx* c, int32_t* ranks, int32_t cap, int32_t* n) {
+  if (!c || !n) return fail(JITC_EINVAL, "jitc_watchdog_failed: null argument");
+  std::lock_guard<std::mutex> lk(c->wmu);
+  *n = (int32_t)c->fired_failed.size();
+  for (int32_t i = 0; i < *n && i < cap && ranks; ++i) ranks[i] = c->fired_failed[i];
+  return JITC_OK;
 }
 
 jitc_status jitc_watchdog_stop(jitc_ctx* c) {

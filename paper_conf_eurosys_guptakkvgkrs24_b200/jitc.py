@@ -119,6 +119,7 @@ def lib() -> ctypes.CDLL:
         "jitc_watchdog_start": ([vp, u32, i32, vp, vp], i32),
         "jitc_watchdog_wait": ([vp, u32, P(i32), P(u64), P(ctypes.c_double), P(ctypes.c_double), P(Stats)], i32),
         "jitc_watchdog_stop": ([vp], i32),
+        "jitc_watchdog_failed": ([vp, P(i32), i32, P(i32)], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -135,8 +136,8 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
             "jitc_inject_release", "jitc_capture_local", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
-            "jitc_watchdog_stop"]
-ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE = 0, 1
+            "jitc_watchdog_stop", "jitc_watchdog_failed"]
+ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE, ON_HANG_COLLECTIVE_CAPTURE = 0, 1, 2
 
 
 def last_error() -> str:
@@ -427,6 +428,12 @@ class Context:
         _check(r, "jitc_watchdog_wait")
         return dict(fired=bool(fired.value), tag=tag.value, waited_ms=waited.value, action_ms=act.value,
                     stats=st.as_dict())
+
+    def watchdog_failed(self) -> List[int]:
+        buf = (ctypes.c_int32 * 64)()
+        n = ctypes.c_int32()
+        _check(self._L.jitc_watchdog_failed(self._h, buf, 64, ctypes.byref(n)), "jitc_watchdog_failed")
+        return list(buf)[:n.value]
 
     def watchdog_stop(self):
         _check(self._L.jitc_watchdog_stop(self._h), "jitc_watchdog_stop")
