@@ -53,34 +53,41 @@ def _run(cmd):
     subprocess.check_call(cmd)
 
 
-def build(force: bool = False, verbose_ptxas: bool = False) -> str:
+def build(force: bool = False, verbose_ptxas: bool = False, sanitize: bool = False) -> str:
+    """sanitize=True builds libjitc_asan.so: host code with AddressSanitizer +
+    UndefinedBehaviorSanitizer (tests/test_asan.py drives it; not the product)."""
     cuda, nccl = _cuda_home(), _nccl_home()
     nvcc = os.path.join(cuda, "bin", "nvcc")
     nccl_lib = os.path.join(nccl, "lib") if os.path.isdir(os.path.join(nccl, "lib")) else "/usr/lib/x86_64-linux-gnu"
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cc")))
     hdrs = sorted(glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(INCLUDE, "*.h")))
+    out = OUT.replace("libjitc.so", "libjitc_asan.so") if sanitize else OUT
+    bdir = BUILD + ("_asan" if sanitize else "")
     newest = max(os.path.getmtime(p) for p in srcs + hdrs + [__file__])
-    if not force and os.path.exists(OUT) and os.path.getmtime(OUT) >= newest:
-        return OUT
-    os.makedirs(BUILD, exist_ok=True)
+    if not force and os.path.exists(out) and os.path.getmtime(out) >= newest:
+        return out
+    os.makedirs(bdir, exist_ok=True)
+    san = ["-Xcompiler", "-fsanitize=address", "-Xcompiler", "-fsanitize=undefined", "-Xcompiler",
+           "-fno-omit-frame-pointer", "-Xcompiler", "-g"] if sanitize else []
     incs = ["-I", INCLUDE, "-I", CSRC, "-I", os.path.join(nccl, "include")]
     objs = []
     for s in srcs:
-        o = os.path.join(BUILD, os.path.basename(s) + ".o")
+        o = os.path.join(bdir, os.path.basename(s) + ".o")
         if s.endswith(".cu"):
             cmd = [nvcc, *ARCH, "-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC", *incs, "-c", s, "-o", o]
             if verbose_ptxas:
                 cmd.insert(1, "-Xptxas=-v")
         else:
-            cmd = [nvcc, "-x", "cu", *ARCH, "-O3", "-std=c++17", "-Xcompiler", "-fPIC,-Wall", *incs, "-c", s, "-o", o]
+            cmd = [nvcc, "-x", "cu", *ARCH, "-O3", "-std=c++17", "-Xcompiler", "-fPIC,-Wall", *san, *incs, "-c", s,
+                   "-o", o]
         _run(cmd)
         objs.append(o)
-    tmp = OUT + ".tmp"
+    tmp = out + ".tmp"
     _run([nvcc, *ARCH, "-shared", "-o", tmp, *objs, "-L", nccl_lib, "-l:libnccl.so.2",
-          f"-Xlinker=-rpath={nccl_lib}", "-cudart", "static"])
-    os.replace(tmp, OUT)
-    return OUT
+          f"-Xlinker=-rpath={nccl_lib}", "-cudart", "static", *san])
+    os.replace(tmp, out)
+    return out
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose_ptxas="-v" in sys.argv)
+    build(force="--force" in sys.argv, verbose_ptxas="-v" in sys.argv, sanitize="--asan" in sys.argv)

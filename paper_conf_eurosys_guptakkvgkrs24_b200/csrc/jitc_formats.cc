@@ -124,7 +124,7 @@ bool parse_blobs(const uint8_t* p, size_t len, std::vector<BlobView>* out, std::
       e.group = t.group;
       e.policy = t.policy;
       e.members.resize(t.n_members);
-      memcpy(e.members.data(), p + q, 4ull * t.n_members);
+      if (t.n_members) memcpy(e.members.data(), p + q, 4ull * t.n_members);
       q += 4ull * t.n_members;
       q = pos + align_up(q - pos, 8);
       bv.topo.push_back(std::move(e));

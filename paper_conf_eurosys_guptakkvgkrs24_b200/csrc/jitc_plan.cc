@@ -200,7 +200,8 @@ extern "C" jitc_status jitc_restore_plan(const void* selection, size_t sel_len, 
   std::vector<PlanOp> ops;
   uint64_t R = 0;
   uint32_t S = 0, J = 0;
-  if (!build_restore_plan(in, &ops, &R, &S, &why, &J)) {
+  // a dropped (OPTIONAL, no candidate) group has nothing to restore: empty plan
+  if (!gs->writers.empty() && !build_restore_plan(in, &ops, &R, &S, &why, &J)) {
     set_error("jitc_restore_plan: " + why);
     return JITC_EINVAL;
   }

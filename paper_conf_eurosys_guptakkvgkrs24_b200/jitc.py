@@ -13,7 +13,9 @@ import struct
 from typing import Dict, List, Optional, Sequence, Tuple
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_PKG, "libjitc.so")
+# JITC_SO overrides the library path (used only by tests/test_asan.py to load
+# the sanitizer build of the same sources).
+SO_PATH = os.environ.get("JITC_SO", os.path.join(_PKG, "libjitc.so"))
 
 OK, EINVAL, ESTATE, ENOMEM, ECUDA, ENCCL = 0, -1, -2, -3, -4, -5
 ELAYOUT, ENOREPLICA, ECONFLICT, ENOCONSISTENT = -6, -7, -8, -9
