@@ -20,8 +20,9 @@ static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelectio
   uint64_t c0, c1;
   shard_range(g.n_c, k, s, &c0, &c1);
   uint64_t b0 = std::min(c0 * g.C, g.L), b1 = std::min(c1 * g.C, g.L);
-  // the lowest writer invalidates the previous commit before any byte changes
-  if (s == 0 && g.img_shm) unlink(gpath(c, g.id, ".commit").c_str());
+  // every writer invalidates the previous commit before it changes any image
+  // byte (whichever writer starts first; unlink is idempotent)
+  if (g.img_shm) unlink(gpath(c, g.id, ".commit").c_str());
   g.commit_priv.clear();
   if (b1 > b0) {
     CU(cudaMemsetAsync(g.d_dig2 + c0, 0, (c1 - c0) * 8, c->s_comp));
@@ -31,7 +32,7 @@ static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelectio
       seg_span(g, b0, b1, &lo, &hi);
       jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, g.img_d, 0), g.d_dig2, b1 - b0);
       if (st) return st;
-      if (stats) stats->rounds += 1;
+      if (stats) stats->rounds += 1, stats->d2h_bytes += b1 - b0;
     } else {
       const uint64_t R = c->slot_bytes;
       const int nslots = (int)std::min<uint64_t>(jitc_ctx::kSlots, c->staging_bytes / R);

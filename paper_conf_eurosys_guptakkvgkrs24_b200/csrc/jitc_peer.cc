@@ -114,7 +114,7 @@ jitc_status jitc_peer_export(jitc_ctx* c, uint32_t group) {
   uint8_t* p = b.data();
   memcpy(p, &h, sizeof h);
   p += sizeof h;
-  memcpy(p, g.fp.data(), 8 * g.n_c);
+  if (g.n_c) memcpy(p, g.fp.data(), 8 * g.n_c);
   p += 8 * g.n_c;
   if (!allocs.empty()) memcpy(p, allocs.data(), sizeof(PeerAlloc) * allocs.size());
   p += sizeof(PeerAlloc) * allocs.size();

@@ -37,19 +37,22 @@ static jitc_status load_manifest(jitc_ctx* c, GroupState& g, ManifestView* mv) {
       h.chunk_bytes != g.C || h.v_star != cr.v_star)
     return fail(JITC_ELAYOUT, "jitc_restore: manifest layout differs from the registered tensors");
   size_t q = sizeof(ManifestHdr);
+  if (4ull * h.k > man.size() - q) return fail(JITC_EINCOMPLETE, "jitc_restore: manifest truncated");
   mv->writers.resize(h.k);
-  memcpy(mv->writers.data(), man.data() + q, 4ull * h.k);
+  if (h.k) memcpy(mv->writers.data(), man.data() + q, 4ull * h.k);
   q = align_up(q + 4ull * h.k, 8);
   size_t t0 = q;
   for (uint32_t i = 0; i < h.n_tensors; ++i) {
     uint16_t ln;
+    if (q + 2 > man.size()) return fail(JITC_EINCOMPLETE, "jitc_restore: manifest truncated");
     memcpy(&ln, man.data() + q, 2);
     q += 2 + ln + 20;
+    if (q > man.size()) return fail(JITC_EINCOMPLETE, "jitc_restore: manifest truncated");
   }
   q = t0 + align_up(q - t0, 8);
   if (q + 8 * (h.n_c + 1) > man.size()) return fail(JITC_EINCOMPLETE, "jitc_restore: manifest truncated");
   mv->d.resize(h.n_c);
-  memcpy(mv->d.data(), man.data() + q, 8 * h.n_c);
+  if (h.n_c) memcpy(mv->d.data(), man.data() + q, 8 * h.n_c);
   memcpy(&mv->root, man.data() + q + 8 * h.n_c, 8);
   if (root_of(h.layout_hash, mv->d.data(), h.n_c) != mv->root)
     return fail(JITC_EINCOMPLETE, "jitc_restore: manifest digests do not chain to its root");
