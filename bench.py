@@ -174,6 +174,8 @@ def run_jitc(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if os.environ.get("JITC_BENCH_SHARE_GPU"):   # functional test of the N>1 path on a 1-GPU box; not a measurement
+        local = 0
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
     torch.cuda.set_device(local)
