@@ -31,6 +31,9 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 HOST_LINK_NOMINAL = 63.0   # PCIe Gen5 x16 GB/s per direction (context)
+# measured on this pool's B200 boxes (profiles/r01_pcie_probe.txt, tools/pcie_probe.cu): the copy-engine
+# limit for 4 GiB transfers, identical for cudaHostAlloc / shm+register / malloc+register and 1-4 streams
+HOST_LINK_MEASURED = {"d2h": 57.2, "h2d": 55.6}
 
 
 def _peaks():
@@ -324,9 +327,11 @@ def run_jitc(args):
             "phases_ms_median": med,
             "capture_GBps": round(L_total / world / (cap_ms * 1e-3) / 1e9, 3),
             "restore_GBps": round(L_total / (res_ms * 1e-3) / 1e9, 3),
-            "host_link_roofline": {"capture_d2h_GBps_nominal": HOST_LINK_NOMINAL,
+            "host_link_roofline": {"nominal_GBps": HOST_LINK_NOMINAL, "measured_GBps": HOST_LINK_MEASURED,
                                    "capture_frac_nominal": round(L_total / world / (med["capture"] * 1e-3) / 1e9 / HOST_LINK_NOMINAL, 3),
-                                   "restore_frac_nominal": round(L_total / world / (res_ms * 1e-3) / 1e9 / HOST_LINK_NOMINAL, 3)},
+                                   "restore_frac_nominal": round(L_total / world / (res_ms * 1e-3) / 1e9 / HOST_LINK_NOMINAL, 3),
+                                   "capture_frac_measured": round(L_total / world / (med["capture"] * 1e-3) / 1e9 / HOST_LINK_MEASURED["d2h"], 3),
+                                   "restore_frac_measured": round(L_total / world / (res_ms * 1e-3) / 1e9 / HOST_LINK_MEASURED["h2d"], 3)},
             "roofline": {"kernel": kinds[dom], "bound": "hbm", "achieved": round(achieved, 1) if achieved else None,
                          "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
                          "traffic": traffic, "peak_source": peak_src,
