@@ -248,6 +248,15 @@ jitc_status jitc_commit(jitc_ctx* ctx, const void* selection, size_t sel_len);
  * watchdog runs with JITC_ON_HANG_LOCAL_CAPTURE. */
 jitc_status jitc_capture_local(jitc_ctx* ctx, jitc_stats* stats);
 
+/* The user's CPU state -- iteration number, RNG state, data-loader position
+ * (save_checkpoint saves "any CPU state") -- as an opaque blob
+ * carried in every group's manifest of the next jitc_commit (covered by the
+ * manifest trailer and the commit record), and read back after a HOST
+ * restore (or on the committing writer) with jitc_get_aux.  cap == 0 =>
+ * only *len. */
+jitc_status jitc_set_aux(jitc_ctx* ctx, const void* data, size_t len);
+jitc_status jitc_get_aux(jitc_ctx* ctx, uint32_t group, void* out, size_t cap, size_t* len);
+
 /* ---- restore ------------------------------------------------------------- */
 /* A9-A11.  HOST: refuses an uncommitted image (JITC_EINCOMPLETE); each comm
  * rank loads chunk range O5(n_c, n, r) H2D, the ranks all-gather the slices

@@ -95,7 +95,8 @@ jitc_status jitc_capture(jitc_ctx* c, const void* selection, size_t sel_len, uin
 }
 
 // ------------------------------------------------------------ commit (manifest, then commit record)
-static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelection& gs, uint64_t v_star) {
+static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelection& gs, uint64_t v_star,
+                                           const std::vector<uint8_t>& aux) {
   std::vector<uint8_t> b;
   ManifestHdr h{};
   h.magic = kMagicManifest;
@@ -132,6 +133,11 @@ static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelec
     shard_range(g.n_c, gs.writers.size(), s, &e.c0, &e.c1);
     put(&e, sizeof e);
   }
+  // the user's CPU state (iteration, RNG, data position: PAPER.md:132), opaque
+  uint64_t aux_len = aux.size();
+  put(&aux_len, 8);
+  if (aux_len) put(aux.data(), aux_len);
+  pad();
   uint64_t tr = manifest_trailer(b.data(), b.size());
   put(&tr, 8);
   return b;
@@ -155,7 +161,7 @@ jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len
     bool writer = std::find(gs->writers.begin(), gs->writers.end(), c->cfg.rank) != gs->writers.end();
     if (!writer) continue;
     if (!g.captured || g.cap_v != sel.v_star) return fail(JITC_ESTATE, "jitc_commit: group not captured at v*");
-    std::vector<uint8_t> man = build_manifest(g, *gs, sel.v_star);
+    std::vector<uint8_t> man = build_manifest(g, *gs, sel.v_star, c->aux);
     CommitRec cr{};
     cr.magic = kMagicCommit;
     cr.group = g.id;
@@ -164,6 +170,7 @@ jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len
     cr.manifest_bytes = man.size();
     g.man_d = g.fp;
     g.man_root = g.fp_root;
+    g.man_aux = c->aux;
     g.has_man = true;
     g.man_priv = man;
     g.commit_priv.assign((uint8_t*)&cr, (uint8_t*)&cr + sizeof cr);

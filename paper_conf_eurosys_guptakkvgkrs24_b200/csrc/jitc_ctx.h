@@ -61,6 +61,7 @@ struct GroupState {
   bool has_man = false;
   std::vector<uint64_t> man_d;
   uint64_t man_root = 0;
+  std::vector<uint8_t> man_aux;  // the user's CPU state carried by the manifest
   // host image
   uint8_t* img_h = nullptr;
   uint8_t* img_d = nullptr;  // device alias of the mapped host image
@@ -138,6 +139,7 @@ struct jitc_ctx {
   int comm_n = 0, comm_rank = -1;
   std::vector<int32_t> comm_job;  // comm rank -> job rank
   std::unique_ptr<IpcComm> ipc;   // IPC transport (instead of `comm`)
+  std::vector<uint8_t> aux;       // user CPU state for the next commit (jitc_set_aux)
   uint64_t* d_small = nullptr;    // 64 B device scratch for size exchange / barrier
   uint32_t* d_work = nullptr;     // K1/K2/K3 batch counters (self-resetting)
   uint64_t* h_small = nullptr;    // pinned

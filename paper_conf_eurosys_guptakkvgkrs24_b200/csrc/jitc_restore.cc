@@ -11,6 +11,7 @@ struct ManifestView {
   std::vector<int32_t> writers;
   std::vector<uint64_t> d;
   uint64_t root = 0;
+  std::vector<uint8_t> aux;
 };
 
 static jitc_status load_manifest(jitc_ctx* c, GroupState& g, ManifestView* mv) {
@@ -56,6 +57,13 @@ static jitc_status load_manifest(jitc_ctx* c, GroupState& g, ManifestView* mv) {
   memcpy(&mv->root, man.data() + q + 8 * h.n_c, 8);
   if (root_of(h.layout_hash, mv->d.data(), h.n_c) != mv->root)
     return fail(JITC_EINCOMPLETE, "jitc_restore: manifest digests do not chain to its root");
+  q += 8 * (h.n_c + 1) + sizeof(ShardEnt) * (uint64_t)h.k;   // skip d[], root and the shard table
+  uint64_t aux_len = 0;
+  if (q + 8 > man.size() - 8) return fail(JITC_EINCOMPLETE, "jitc_restore: manifest truncated");
+  memcpy(&aux_len, man.data() + q, 8);
+  q += 8;
+  if (aux_len > man.size() - 8 - q) return fail(JITC_EINCOMPLETE, "jitc_restore: manifest truncated");
+  mv->aux.assign(man.data() + q, man.data() + q + aux_len);
   return JITC_OK;
 }
 
@@ -262,6 +270,7 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
   g.man_d = mv.d;
   g.man_root = mv.root;
   g.has_man = true;
+  g.man_aux = mv.aux;
   if (stats) stats->image_bytes += g.L;
   return JITC_OK;
 }
@@ -402,6 +411,26 @@ jitc_status jitc_restore(jitc_ctx* c, uint32_t group, int32_t mode, const void* 
   CU(cudaEventRecord(c->ev_t1, c->s_comp));
   CU(cudaEventSynchronize(c->ev_t1));
   finish_stats(c, t, stats, true);
+  return JITC_OK;
+}
+
+// ------------------------------------------------------------ user CPU state
+jitc_status jitc_set_aux(jitc_ctx* c, const void* data, size_t len) {
+  if (!c || (len && !data)) return fail(JITC_EINVAL, "jitc_set_aux: bad argument");
+  c->aux.assign(static_cast<const uint8_t*>(data), static_cast<const uint8_t*>(data) + len);
+  return JITC_OK;
+}
+
+jitc_status jitc_get_aux(jitc_ctx* c, uint32_t group, void* out, size_t cap, size_t* len) {
+  if (!c || !len) return fail(JITC_EINVAL, "jitc_get_aux: bad argument");
+  auto it = c->groups.find(group);
+  if (it == c->groups.end() || !it->second.held || !it->second.has_man)
+    return fail(JITC_ESTATE, "jitc_get_aux: no restored / committed manifest for the group");
+  const std::vector<uint8_t>& a = it->second.man_aux;
+  *len = a.size();
+  if (cap == 0) return JITC_OK;
+  if (cap < a.size() || (!out && !a.empty())) return fail(JITC_EINVAL, "jitc_get_aux: buffer too small");
+  if (!a.empty()) memcpy(out, a.data(), a.size());
   return JITC_OK;
 }
 

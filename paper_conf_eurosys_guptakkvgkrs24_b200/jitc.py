@@ -113,6 +113,8 @@ def lib() -> ctypes.CDLL:
         "jitc_inject_release": ([u32], i32),
         "jitc_watch_event": ([vp, vp, u64], i32),
         "jitc_capture_local": ([vp, P(Stats)], i32),
+        "jitc_set_aux": ([vp, vp, sz], i32),
+        "jitc_get_aux": ([vp, u32, vp, sz, P(sz)], i32),
         "jitc_peer_export": ([vp, u32], i32),
         "jitc_restore_pull": ([vp, u32, vp, sz, P(Stats)], i32),
         "jitc_persist": ([vp, u32, ctypes.c_char_p, P(Stats)], i32),
@@ -137,7 +139,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_select_consistent_replica", "jitc_capture", "jitc_commit", "jitc_restore", "jitc_verify",
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
-            "jitc_inject_release", "jitc_capture_local", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
+            "jitc_inject_release", "jitc_capture_local", "jitc_set_aux", "jitc_get_aux", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop", "jitc_watchdog_failed"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE, ON_HANG_COLLECTIVE_CAPTURE = 0, 1, 2
 
@@ -380,6 +382,17 @@ class Context:
         st = Stats()
         _check(self._L.jitc_stage_in(self._h, group, directory.encode(), ctypes.byref(st)), "jitc_stage_in")
         return st.as_dict()
+
+    def set_aux(self, data: bytes):
+        """CPU state (iteration, RNG, ...) to carry in the next commit's manifests."""
+        _check(self._L.jitc_set_aux(self._h, data, len(data)), "jitc_set_aux")
+
+    def get_aux(self, group: int) -> bytes:
+        n = ctypes.c_size_t()
+        _check(self._L.jitc_get_aux(self._h, group, None, 0, ctypes.byref(n)), "jitc_get_aux")
+        buf = ctypes.create_string_buffer(max(n.value, 1))
+        _check(self._L.jitc_get_aux(self._h, group, buf, n.value, ctypes.byref(n)), "jitc_get_aux")
+        return buf.raw[:n.value]
 
     def commit(self, selection: bytes):
         _check(self._L.jitc_commit(self._h, selection, len(selection)), "jitc_commit")

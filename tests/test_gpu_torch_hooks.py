@@ -71,6 +71,10 @@ def test_hooks_selection_restore_and_loss_match(J):
         assert st == J.OK and s["v_star"] == 3
         assert s["groups"][0]["writers"] == [0] and s["groups"][0]["excluded"] == [(1, J.DIRTY)]
         ctxs[0].capture(sel)
+        import pickle
+        cpu_state = {"version": 3, "adam_steps": [opts[0].state[p]["step"].item() for p in reps[0].parameters()],
+                     "torch_rng": torch.get_rng_state()}
+        ctxs[0].set_aux(pickle.dumps(cpu_state))             # the user's CPU state rides in the manifest
         ctxs[0].commit(sel)
         # a replacement for rank 1: fresh model + optimizer, restored from the image
         m2 = _model(99)
@@ -84,10 +88,12 @@ def test_hooks_selection_restore_and_loss_match(J):
         torch.cuda.synchronize()
         for (n, a), b in zip(reps[0].state_dict().items(), m2.state_dict().values()):
             assert torch.equal(a, b), n
-        for p0, p2 in zip(reps[0].parameters(), m2.parameters()):
+        restored_cpu = pickle.loads(ctx2.get_aux(0))
+        assert restored_cpu["version"] == 3 and torch.equal(restored_cpu["torch_rng"], cpu_state["torch_rng"])
+        for i, (p0, p2) in enumerate(zip(reps[0].parameters(), m2.parameters())):
             for k in ("exp_avg", "exp_avg_sq"):
                 assert torch.equal(opts[0].state[p0][k], o2.state[p2][k])
-            o2.state[p2]["step"] = opts[0].state[p0]["step"].clone()   # a CPU scalar: the user's CPU state (R1)
+            o2.state[p2]["step"].fill_(restored_cpu["adam_steps"][i])   # CPU scalar from the manifest's aux
         # training continues: the losses match bit for bit
         for x, y in data[3:]:
             la, lb = _step(reps[0], opts[0], x, y), _step(m2, o2, x, y)
