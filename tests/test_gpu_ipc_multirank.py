@@ -81,6 +81,35 @@ if phase == "host":
     res = ctx.restore(J.ALL_GROUPS, J.HOST)             # 1/n H2D + peers' slices over IPC, fused into K3
     check(ctx, sts, {{0, 1, 2}})
     print("host ok", cap["image_bytes"], res["h2d_bytes"], res["p2p_bytes"], flush=True)
+elif phase in ("w0", "repl", "dirty"):
+    # rank 0 healthy; rank 1 replaced; rank 2 alive but DIRTY with a half-applied
+    # update: both non-writers are repaired from rank 0 (SURVEY O8 destinations)
+    ctx, sts = make_ctx(shm + "/comm3", scramble=(phase == "repl"))
+    if phase == "dirty":
+        g0 = groups[0]
+        for i in range(0, len(g0.tensors), 2):
+            t = g0.tensors[i]
+            J.inject_update(sts[0].ptrs[i], 0, t.nbytes // 4, t.gen_id, 34)
+        torch.cuda.synchronize()
+        ctx.mark(0, 33, J.DIRTY)
+    if phase != "repl":
+        open(f"{{shm}}/blob3.{{rank}}", "wb").write(ctx.fingerprint())
+    t0 = time.time()
+    while not all(os.path.exists(f"{{shm}}/blob3.{{r}}") for r in (0, 2)) and time.time() - t0 < 120:
+        time.sleep(0.02)
+    time.sleep(0.2)
+    blobs = b"".join(open(f"{{shm}}/blob3.{{r}}", "rb").read() for r in (0, 2))
+    st_, sel = J.select_consistent_replica(blobs, [0, 2])
+    assert st_ == J.OK, J.parse_selection(sel)
+    gsel = {{g["group"]: g for g in J.parse_selection(sel)["groups"]}}
+    assert gsel[0]["writers"] == [0] and gsel[0]["excluded"] == [(2, J.DIRTY)], gsel[0]
+    ctx.restore(J.ALL_GROUPS, J.PEER, sel)
+    if phase == "repl":
+        check(ctx, sts, {{0, 1, 2}})
+    elif phase == "dirty":                       # repaired in group 0; a writer of group 1
+        assert gsel[1]["writers"] == [0, 2]
+        check(ctx, sts, {{0}})
+    print(phase, "ok", flush=True)
 elif phase in ("writer", "replacement"):
     # rank 1 died; ranks 0 and 2 keep their state, a replacement process joins
     ctx, sts = make_ctx(shm + "/comm2", scramble=(phase == "replacement"))
@@ -135,5 +164,15 @@ def test_ipc_multirank_peer_restore_of_replacement():
     try:
         outs = _spawn(shm, 3, {0: "writer", 1: "replacement", 2: "writer"})
         assert "peer ok" in outs[1] and "writer ok" in outs[0] and "writer ok" in outs[2], outs
+    finally:
+        shutil.rmtree(shm, ignore_errors=True)
+
+
+def test_ipc_peer_repairs_replacement_and_dirty_member():
+    shm = f"/dev/shm/jitc-ipc-{os.getpid()}-{uuid.uuid4().hex[:8]}"
+    os.makedirs(shm)
+    try:
+        outs = _spawn(shm, 3, {0: "w0", 1: "repl", 2: "dirty"})
+        assert "w0 ok" in outs[0] and "repl ok" in outs[1] and "dirty ok" in outs[2], outs
     finally:
         shutil.rmtree(shm, ignore_errors=True)
