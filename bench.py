@@ -207,6 +207,7 @@ def run_jitc(args):
     for g in w.groups:
         if rank not in g.members:
             ctx.declare_group(g.group, g.policy, g.members)
+    t_comm = time.perf_counter()
     if world > 1:
         if args.transport == "nccl":
             uid = [J.get_unique_id() if rank == 0 else None]
@@ -214,6 +215,7 @@ def run_jitc(args):
             ctx.comm_init(uid[0], world, rank)
         else:   # intra-node CUDA IPC transport (fresh directory per communicator)
             ctx.comm_init_ipc(f"{shm}-comm", world, rank)
+    comm_init_ms = (time.perf_counter() - t_comm) * 1e3
     torch.cuda.synchronize()
     setup_s = time.perf_counter() - t_setup
 
@@ -320,6 +322,7 @@ def run_jitc(args):
             "config": {"workload": w.name, "image_bytes": L_total, "tensors": sum(len(g.tensors) for g in w.groups_of(rank)),
                        "writers_k": world, "restore_mode": "HOST", "image": "shared /dev/shm",
                        "transport": args.transport if world > 1 else None,
+                       "comm_init_ms": round(comm_init_ms, 1) if world > 1 else None,
                        "zero_copy": bool(args.zero_copy), "chunk_bytes": 1 << 20,
                        "staging_mib": args.staging, "slot_mib": args.slot,
                        "l2": f"state {L_total / 1e9:.1f} GB >> 126 MB L2; no flush needed", "setup_s": round(setup_s, 1)},

@@ -70,6 +70,7 @@ static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelectio
 }
 
 jitc_status jitc_capture(jitc_ctx* c, const void* selection, size_t sel_len, uint32_t group, jitc_stats* stats) {
+  NvtxRange nvtx_("jitc_capture");
   if (!c) return fail(JITC_EINVAL, "jitc_capture: null ctx");
   Selection sel;
   std::string why;
@@ -185,6 +186,7 @@ jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len
 }
 
 jitc_status jitc_commit(jitc_ctx* c, const void* selection, size_t sel_len) {
+  NvtxRange nvtx_("jitc_commit");
   return commit_impl(c, selection, sel_len, true);
 }
 

@@ -407,6 +407,7 @@ static RecordHdr record_of(const jitc_ctx* c, const GroupState& g) {
 }
 
 jitc_status jitc_fingerprint(jitc_ctx* c, uint32_t group, void* blob, size_t cap, size_t* len) {
+  NvtxRange nvtx_("jitc_fingerprint");
   if (!c || !len) return fail(JITC_EINVAL, "jitc_fingerprint: null argument");
   CU(cudaSetDevice(c->device));
   std::vector<GroupState*> sel;
@@ -435,6 +436,7 @@ jitc_status jitc_fingerprint(jitc_ctx* c, uint32_t group, void* blob, size_t cap
 
 // ------------------------------------------------------------ record exchange (C1)
 jitc_status jitc_exchange_records(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len) {
+  NvtxRange nvtx_("jitc_exchange_records");
   if (!c || !mine || !all_len || len < sizeof(BlobHdr)) return fail(JITC_EINVAL, "jitc_exchange_records: bad argument");
   if (c->ipc) return ipc_exchange(c, mine, len, all, cap, all_len);
   if (!c->comm) {

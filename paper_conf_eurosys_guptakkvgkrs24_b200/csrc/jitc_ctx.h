@@ -26,6 +26,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "jitc_internal.h"
 
 
@@ -202,6 +204,12 @@ struct CallTimer {
     c->kernel_ms_in_call = 0;
     c->kev_used = 0;
   }
+};
+
+// NVTX range for Nsight timelines (header-only NVTX3; a no-op without a tool attached)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
 };
 
 // Kernel launch with optional event bracketing (JITC_F_TIME_KERNELS).

@@ -126,6 +126,7 @@ jitc_status jitc_peer_export(jitc_ctx* c, uint32_t group) {
 }
 
 jitc_status jitc_restore_pull(jitc_ctx* c, uint32_t group, const void* selection, size_t sel_len, jitc_stats* stats) {
+  NvtxRange nvtx_("jitc_restore_pull");
   if (!c) return fail(JITC_EINVAL, "jitc_restore_pull: null ctx");
   Selection sel;
   std::string why;

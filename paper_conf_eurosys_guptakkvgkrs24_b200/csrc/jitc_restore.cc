@@ -379,6 +379,7 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
 
 jitc_status jitc_restore(jitc_ctx* c, uint32_t group, int32_t mode, const void* selection, size_t sel_len,
                          jitc_stats* stats) {
+  NvtxRange nvtx_(mode == JITC_RESTORE_HOST ? "jitc_restore(HOST)" : "jitc_restore(PEER)");
   if (!c) return fail(JITC_EINVAL, "jitc_restore: null ctx");
   if (mode != JITC_RESTORE_HOST && mode != JITC_RESTORE_PEER) return fail(JITC_EINVAL, "jitc_restore: bad mode");
   Selection sel;
@@ -436,6 +437,7 @@ jitc_status jitc_get_aux(jitc_ctx* c, uint32_t group, void* out, size_t cap, siz
 
 // ------------------------------------------------------------ verify (A12)
 jitc_status jitc_verify(jitc_ctx* c, uint32_t group, const void* expected, size_t len, uint64_t* first_bad) {
+  NvtxRange nvtx_("jitc_verify");
   if (!c) return fail(JITC_EINVAL, "jitc_verify: null ctx");
   if (first_bad) *first_bad = UINT64_MAX;
   auto it = c->groups.find(group);
