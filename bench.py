@@ -179,6 +179,9 @@ def run_jitc(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if os.environ.get("JITC_BENCH_SHARE_GPU"):   # functional test of the N>1 path on a 1-GPU box; not a measurement
         local = 0
+        if args.transport == "nccl":   # NCCL refuses two ranks per GPU on one host: one fake host per rank
+            os.environ.update(NCCL_HOSTID=f"jitc-bench-host-{rank}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
+                              NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0")
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
     torch.cuda.set_device(local)

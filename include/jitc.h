@@ -34,9 +34,10 @@
  *    watchdog thread (no callbacks, so no GIL).
  *  - Collective calls (every member of the library communicator must call):
  *    jitc_comm_init, jitc_comm_shrink, jitc_exchange_records, jitc_commit,
- *    jitc_restore.  Local: register, declare_group, mark, fingerprint,
- *    capture, verify.  Pure (no ctx, no GPU): jitc_layout, jitc_shard_range,
- *    jitc_select_consistent_replica, jitc_restore_plan.
+ *    jitc_restore, jitc_capture_fanout.  Local: register, declare_group,
+ *    attach_image, mark, fingerprint, capture, verify.  Pure (no ctx, no
+ *    GPU): jitc_layout, jitc_shard_range, jitc_select_consistent_replica,
+ *    jitc_restore_plan, jitc_capture_plan.
  *  - No CPU fallback: if the device or the sm_100a kernels are unavailable
  *    the call fails with JITC_ECUDA.
  *  - Binary formats (record blob, selection, manifest, commit record) are
@@ -239,6 +240,33 @@ jitc_status jitc_capture(jitc_ctx* ctx, const void* selection, size_t sel_len, u
  * the lowest-rank writer of each group writes it. */
 jitc_status jitc_commit(jitc_ctx* ctx, const void* selection, size_t sel_len);
 
+/* Capture with NVLink fan-out.  Capture is
+ * bound by each writer's host link (PCIe), so a group with few writers --
+ * k = 1 for the TP partition whose other replica died (C5), a ZeRO shard
+ * (C4) -- would leave the other GPUs' links idle.  Collective over the
+ * communicator (every comm rank calls it, with the same arguments).  For
+ * `group` (or every group of the selection, in increasing id, with
+ * JITC_ALL_GROUPS): writer s still packs and re-digests exactly its O5(n_c,
+ * k, s) shard (JITC_EUNSTABLE as for jitc_capture), but the image is D2H'd
+ * in m lanes, lane q = O5(n_c, m, q) by the q-th of `movers` (job ranks,
+ * taken in sorted order, all in the communicator); the part of shard s that
+ * falls in another mover's lane is sent to it over NVLink (NCCL send/recv,
+ * or with the IPC transport a peer-to-peer copy out of the writer's
+ * staging) and that mover D2Hs it with its own copy engine and PCIe link.
+ * Every mover must hold the group's host image: its own (a member) or one
+ * attached with jitc_attach_image.  The image bytes, the manifest and the
+ * shard table are exactly those of jitc_capture; jitc_commit follows as
+ * usual.  Needs a shared image_dir. */
+jitc_status jitc_capture_fanout(jitc_ctx* ctx, const void* selection, size_t sel_len, uint32_t group,
+                                const int32_t* movers, int32_t n_movers, jitc_stats* stats);
+/* Steady-state preparation of a fan-out mover for a group it does not hold
+ * (declared with jitc_declare_group): maps image_dir/g<group>.img, sized for
+ * an image of `image_bytes` (the L that jitc_register of the group's members
+ * returns), and pins it, so that jitc_capture_fanout neither maps nor pins in
+ * the failure path.  JITC_EINVAL if the group is held or undeclared, or the
+ * context has no image_dir. */
+jitc_status jitc_attach_image(jitc_ctx* ctx, uint32_t group, uint64_t image_bytes);
+
 /* Local (non-collective) capture of every held group by this rank alone:
  * fingerprint -> select over its own record -> capture (k = 1) -> commit.
  * The paper's user-level protocol in which each healthy rank saves its own
@@ -308,6 +336,13 @@ jitc_status jitc_restore_plan(const void* selection, size_t sel_len, uint32_t gr
                               const int32_t* comm_job_ranks, int32_t n, int32_t comm_rank,
                               uint64_t staging_bytes, uint64_t slot_bytes, void* plan, size_t cap,
                               size_t* len);
+
+/* The round schedule jitc_capture_fanout executes for `group` on comm rank
+ * `comm_rank` (same header and 48-B operations as jitc_restore_plan; kinds
+ * 3 PACK, 4 SEND, 5 RECV, 9 D2H).  Pure.  cap == 0 => only *len. */
+jitc_status jitc_capture_plan(const void* selection, size_t sel_len, uint32_t group, const int32_t* movers,
+                              int32_t n_movers, const int32_t* comm_job_ranks, int32_t n, int32_t comm_rank,
+                              uint64_t staging_bytes, uint64_t slot_bytes, void* plan, size_t cap, size_t* len);
 
 /* ---- durable tier (NEXT-4; §6.3) ---------------------- */
 /* Streams the committed host image of `group` to `dir` (parallel O_DIRECT

@@ -48,7 +48,7 @@ static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelectio
         if (st) return st;
         CU(cudaEventRecord(c->ev_ready[sl], c->s_comp));
         CU(cudaStreamWaitEvent(c->s_copy, c->ev_ready[sl], 0));
-        CU(cudaMemcpyAsync(g.img_h + a, slot, b - a, cudaMemcpyDeviceToHost, c->s_copy));
+        CU(copy_pieces(c, g.img_h + a, slot, b - a, cudaMemcpyDeviceToHost, c->s_copy));
         CU(cudaEventRecord(c->ev_free[sl], c->s_copy));
       }
       if (stats) stats->rounds += j;
@@ -88,6 +88,190 @@ jitc_status jitc_capture(jitc_ctx* c, const void* selection, size_t sel_len, uin
     if (!gs) return fail(JITC_ELAYOUT, "jitc_capture: group missing from selection");
     jitc_status st = capture_group(c, g, *gs, sel.v_star, stats);
     if (st) return st;
+  }
+  CU(cudaEventRecord(c->ev_t1, c->s_comp));
+  CU(cudaEventSynchronize(c->ev_t1));
+  finish_stats(c, t, stats, true);
+  return JITC_OK;
+}
+
+// ------------------------------------------------------------ capture with NVLink fan-out
+// Executes build_capture_plan (jitc_plan.cc) for one group, round by round:
+// the writer's K2 packs and the transfers on the compute stream, the D2H of
+// every block this rank moves on the copy stream; slot reuse is ordered by
+// the ready/free events.  NCCL: grouped send/recv per round.  IPC: a writer
+// posts its round (stream-ordered counter write), a mover copies the block
+// out of the writer's staging (peer-to-peer over NVLink) into its own and
+// posts "consumed"; a writer refills a slot only after its readers consumed
+// the round that last used it, and returns only after they read every round.
+static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection& gs, uint64_t v_star,
+                                const int32_t* movers, int32_t n_movers, uint64_t gen, jitc_stats* stats) {
+  PlanInput in;
+  std::string why;
+  if (!capture_plan_input(gs, movers, n_movers, c->comm_job.data(), c->comm_n, c->comm_rank, c->staging_bytes,
+                          c->slot_bytes, &in, &why))
+    return fail(JITC_EINVAL, "jitc_capture_fanout: " + why);
+  std::vector<PlanOp> ops;
+  uint64_t R = 0;
+  uint32_t S = 0, J = 0;
+  if (!build_capture_plan(in, &ops, &R, &S, &why, &J)) return fail(JITC_ENOMEM, "jitc_capture_fanout: " + why);
+  if (S > (uint32_t)jitc_ctx::kSlots) return fail(JITC_EINVAL, "jitc_capture_fanout: too many slots");
+  const int me = c->comm_rank;
+  const auto wit = std::find(in.writers.begin(), in.writers.end(), me);
+  const bool is_writer = wit != in.writers.end();
+  const bool is_mover = std::find(in.movers.begin(), in.movers.end(), me) != in.movers.end();
+  if (!is_writer && !is_mover) return JITC_OK;
+  uint64_t c0 = 0, c1 = 0;
+  if (is_writer) {
+    if (!g.held) return fail(JITC_ESTATE, "jitc_capture_fanout: writer does not hold the group");
+    if (!g.has_fp) return fail(JITC_ESTATE, "jitc_capture_fanout: group " + std::to_string(g.id) + " not fingerprinted");
+    if (gs.layout_hash != g.layout_hash || gs.n_c != g.n_c || gs.image_bytes != g.L)
+      return fail(JITC_ELAYOUT, "jitc_capture_fanout: selection layout differs from the registered one");
+    if (g.fp_version != v_star || g.fp_root != gs.root || g.fp_phase != JITC_PHASE_CLEAN)
+      return fail(JITC_ESTATE, "jitc_capture_fanout: this rank's fingerprint is not the selected candidate");
+    shard_range(g.n_c, in.writers.size(), (uint64_t)(wit - in.writers.begin()), &c0, &c1);
+    if (g.img_shm) unlink(gpath(c, g.id, ".commit").c_str());  // invalidate before any image byte changes
+    g.commit_priv.clear();
+    if (c1 > c0) CU(cudaMemsetAsync(g.d_dig2 + c0, 0, (c1 - c0) * 8, c->s_comp));
+  }
+  bool moves = false;
+  for (const PlanOp& op : ops) moves |= op.kind == kOpD2H;
+  if (moves && (!g.img_h || !g.img_shm || g.L != gs.image_bytes))
+    return fail(JITC_EINVAL, "jitc_capture_fanout: mover has no host image of group " + std::to_string(g.id) +
+                                 " (jitc_attach_image)");
+  IpcComm* ic = c->ipc.get();
+  const uint32_t gsl = ic ? group_slot(c, g.id) : 0;
+  const int my_slot = ic ? ic->slot[me] : 0;
+  std::vector<int> readers;  // movers that receive from me (IPC slot reuse)
+  for (const PlanOp& op : ops)
+    if (op.kind == kOpSend && std::find(readers.begin(), readers.end(), op.peer) == readers.end())
+      readers.push_back(op.peer);
+  bool used[jitc_ctx::kSlots] = {false};
+  size_t i = 0;
+  uint32_t rounds = 0;
+  for (uint32_t j = 0; j < J; ++j) {
+    size_t e = i;
+    while (e < ops.size() && ops[e].round == j) ++e;
+    const uint32_t sl = j % S;
+    const uint64_t seq = (gen << 24) | (j + 1);
+    if (e > i) ++rounds;
+    if (e > i && used[sl]) CU(cudaStreamWaitEvent(c->s_comp, c->ev_free[sl], 0));
+    bool packs = false;
+    for (size_t q = i; q < e; ++q) packs |= ops[q].kind == kOpPack;
+    // IPC: my readers must have consumed the round that last used this slot
+    if (ic && packs && j >= S)
+      for (int r : readers) {
+        jitc_status st = ipc_wait(&ic->ctl->cap_consumed[ic->slot[r]][gsl], seq - S, "a mover to consume a round");
+        if (st) return st;
+      }
+    // 1. K2: pack my block (re-digest into d_dig2)
+    for (size_t q = i; q < e; ++q) {
+      const PlanOp& op = ops[q];
+      if (op.kind != kOpPack) continue;
+      uint32_t lo, hi;
+      seg_span(g, op.a, op.b, &lo, &hi);
+      jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, c->staging + op.off, op.a), g.d_dig2, op.b - op.a);
+      if (st) return st;
+    }
+    // 2. NVLink: writer -> mover
+    if (ic) {
+      if (is_writer) {
+        jitc_status st = ipc_post(c, &ic->ctl->cap_posted[my_slot][gsl], seq, c->s_comp);
+        if (st) return st;
+      }
+      bool recv = false;
+      for (size_t q = i; q < e; ++q) {
+        const PlanOp& op = ops[q];
+        if (op.kind != kOpRecv) continue;
+        recv = true;
+        jitc_status st = ipc_wait(&ic->ctl->cap_posted[ic->slot[op.peer]][gsl], seq, "a writer to post a round");
+        if (st) return st;
+        CU(cudaMemcpyAsync(c->staging + op.off, ic->peer_staging[op.peer] + op.off, op.bytes, cudaMemcpyDefault,
+                           c->s_comp));
+        if (stats) stats->p2p_bytes += op.bytes;
+      }
+      if (recv || is_mover) {
+        jitc_status st = ipc_post(c, &ic->ctl->cap_consumed[my_slot][gsl], seq, c->s_comp);
+        if (st) return st;
+      }
+    } else {
+      bool p2p = false;
+      for (size_t q = i; q < e; ++q) p2p |= ops[q].kind == kOpSend || ops[q].kind == kOpRecv;
+      if (p2p) {
+        NC(ncclGroupStart());
+        for (size_t q = i; q < e; ++q) {
+          const PlanOp& op = ops[q];
+          if (op.kind == kOpSend) NC(ncclSend(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+          if (op.kind == kOpRecv) NC(ncclRecv(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
+          if (stats) stats->p2p_bytes += op.bytes;
+        }
+        NC(ncclGroupEnd());
+      }
+    }
+    // 3. D2H of every block of my lane on the copy stream
+    if (e > i) {
+      CU(cudaEventRecord(c->ev_ready[sl], c->s_comp));
+      CU(cudaStreamWaitEvent(c->s_copy, c->ev_ready[sl], 0));
+      for (size_t q = i; q < e; ++q) {
+        const PlanOp& op = ops[q];
+        if (op.kind != kOpD2H) continue;
+        CU(copy_pieces(c, g.img_h + op.a, c->staging + op.off, op.bytes, cudaMemcpyDeviceToHost, c->s_copy));
+        if (stats) stats->d2h_bytes += op.bytes;
+      }
+      CU(cudaEventRecord(c->ev_free[sl], c->s_copy));
+      used[sl] = true;
+    }
+    i = e;
+  }
+  CU(cudaEventRecord(c->ev_join, c->s_copy));
+  CU(cudaStreamWaitEvent(c->s_comp, c->ev_join, 0));
+  if (is_writer && c1 > c0) CU(cudaMemcpyAsync(c->h_dig, g.d_dig2 + c0, (c1 - c0) * 8, cudaMemcpyDeviceToHost, c->s_comp));
+  CU(cudaStreamSynchronize(c->s_comp));
+  // IPC: my staging may be reused once this call returns -- wait for my readers
+  if (ic && !readers.empty())
+    for (int r : readers) {
+      jitc_status st = ipc_wait(&ic->ctl->cap_consumed[ic->slot[r]][gsl], (gen << 24) | J, "a mover to finish");
+      if (st) return st;
+    }
+  if (stats) stats->rounds += rounds;
+  if (!is_writer) return JITC_OK;
+  for (uint64_t ch = c0; ch < c1; ++ch)
+    if (c->h_dig[ch - c0] != g.fp[ch])
+      return fail(JITC_EUNSTABLE, "jitc_capture_fanout: group " + std::to_string(g.id) + " chunk " +
+                                      std::to_string(ch) + " changed between fingerprint and capture");
+  g.captured = true;
+  g.cap_v = v_star;
+  if (stats) stats->image_bytes += std::min(c1 * g.C, g.L) - std::min(c0 * g.C, g.L);
+  return JITC_OK;
+}
+
+jitc_status jitc_capture_fanout(jitc_ctx* c, const void* selection, size_t sel_len, uint32_t group,
+                                const int32_t* movers, int32_t n_movers, jitc_stats* stats) {
+  NvtxRange nvtx_("jitc_capture_fanout");
+  if (!c || n_movers <= 0 || !movers) return fail(JITC_EINVAL, "jitc_capture_fanout: bad argument");
+  if (!has_comm(c)) return fail(JITC_ESTATE, "jitc_capture_fanout: needs a communicator");
+  if (c->image_dir.empty()) return fail(JITC_EINVAL, "jitc_capture_fanout: needs a shared image_dir");
+  Selection sel;
+  std::string why;
+  if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
+    return fail(JITC_EINVAL, "jitc_capture_fanout: " + why);
+  if (sel.status != JITC_OK) return fail(sel.status, "jitc_capture_fanout: selection status is not OK");
+  CU(cudaSetDevice(c->device));
+  if (stats) memset(stats, 0, sizeof *stats), stats->first_bad_chunk = -1;
+  CallTimer t(c);
+  // every comm rank advances the generation once per call (collective)
+  const uint64_t gen = c->ipc ? ++c->ipc->cap_gen : 0;
+  CU(cudaEventRecord(c->ev_t0, c->s_comp));
+  for (const GroupSelection& gs : sel.groups) {  // increasing group id on every rank
+    if (group != JITC_ALL_GROUPS && gs.group != group) continue;
+    if (gs.writers.empty()) continue;  // dropped OPTIONAL group
+    auto it = c->groups.find(gs.group);
+    if (it == c->groups.end()) return fail(JITC_ELAYOUT, "jitc_capture_fanout: group unknown to this rank");
+    jitc_status st = fanout_group(c, it->second, gs, sel.v_star, movers, n_movers, gen, stats);
+    if (st) {
+      harvest(c);
+      return st;
+    }
   }
   CU(cudaEventRecord(c->ev_t1, c->s_comp));
   CU(cudaEventSynchronize(c->ev_t1));

@@ -79,6 +79,8 @@ jitc_status jitc_create(const jitc_config* cfg, jitc_ctx** out) {
   while (slot > C && slot * 2 > c->staging_bytes) slot = std::max<uint64_t>(slot / 2 / C * C, C);
   if (slot > c->staging_bytes) return fail(JITC_EINVAL, "jitc_create: staging smaller than one chunk");
   c->slot_bytes = slot;
+  c->copy_piece = kDefaultCopyPiece;
+  if (const char* e = getenv("JITC_COPY_PIECE_MB")) c->copy_piece = strtoull(e, nullptr, 10) << 20;
   for (int i = 0; i < jitc_ctx::kSlots; ++i) {
     CU(cudaEventCreateWithFlags(&c->ev_ready[i], cudaEventDisableTiming));
     CU(cudaEventCreateWithFlags(&c->ev_free[i], cudaEventDisableTiming));
@@ -171,6 +173,46 @@ static jitc_status declare(jitc_ctx* c, uint32_t group, int32_t policy, const in
   return JITC_OK;
 }
 
+// Maps image_dir/g<group>.img (g.img_bytes) shared and pins it (mapped,
+// portable).  Several ranks of a box register the same image.  Concurrent
+// cudaHostRegister calls that fault the same fresh tmpfs pages in fail
+// (error 304, measured with >= 8 GiB images: tools/pin_probe2.py), so the
+// pages are allocated up front (posix_fallocate, idempotent) and the
+// registration itself is serialised with an exclusive flock on the file.
+static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::string& who) {
+  mkdir(c->image_dir.c_str(), 0700);
+  g.img_path = gpath(c, g.id, ".img");
+  int fd = open(g.img_path.c_str(), O_RDWR | O_CREAT, 0600);
+  if (fd < 0) return fail(JITC_EIO, who + ": open " + g.img_path + ": " + strerror(errno));
+  flock(fd, LOCK_EX);
+  struct stat sb;
+  int err = 0;
+  if (fstat(fd, &sb) != 0 || ((uint64_t)sb.st_size != g.img_bytes && ftruncate(fd, (off_t)g.img_bytes) != 0))
+    err = errno ? errno : EIO;
+  if (!err) err = posix_fallocate(fd, 0, (off_t)g.img_bytes);
+  if (err) {
+    flock(fd, LOCK_UN);
+    close(fd);
+    return fail(JITC_EIO, who + ": sizing " + g.img_path + ": " + strerror(err));
+  }
+  void* p = mmap(nullptr, g.img_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  if (p == MAP_FAILED) {
+    flock(fd, LOCK_UN);
+    close(fd);
+    return fail(JITC_EIO, who + ": mmap " + g.img_path + ": " + strerror(errno));
+  }
+  cudaError_t e = cudaHostRegister(p, g.img_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+  flock(fd, LOCK_UN);
+  close(fd);
+  if (e != cudaSuccess) {
+    munmap(p, g.img_bytes);
+    return fail(JITC_ENOMEM, who + ": cudaHostRegister: " + cudaGetErrorString(e));
+  }
+  g.img_h = (uint8_t*)p;
+  g.img_shm = true;
+  return JITC_OK;
+}
+
 jitc_status jitc_declare_group(jitc_ctx* c, uint32_t group, int32_t policy, const int32_t* members,
                                int32_t n_members) {
   if (!c) return fail(JITC_EINVAL, "jitc_declare_group: null ctx");
@@ -234,41 +276,8 @@ jitc_status jitc_register(jitc_ctx* c, uint32_t group, int32_t policy, const int
   // host image: shared /dev/shm file (survives the process) or private pinned
   g.img_bytes = std::max<uint64_t>(align_up(g.L, 4096), 4096);
   if (!c->image_dir.empty()) {
-    mkdir(c->image_dir.c_str(), 0700);
-    g.img_path = gpath(c, group, ".img");
-    int fd = open(g.img_path.c_str(), O_RDWR | O_CREAT, 0600);
-    if (fd < 0) return fail(JITC_EIO, "jitc_register: open " + g.img_path + ": " + strerror(errno));
-    // Several ranks of a box register the same image.  Concurrent
-    // cudaHostRegister calls that fault the same fresh tmpfs pages in fail
-    // (error 304, measured with >= 8 GiB images: tools/pin_probe2.py), so
-    // the pages are allocated up front (posix_fallocate, idempotent) and the
-    // registration itself is serialised with an exclusive flock on the file.
-    flock(fd, LOCK_EX);
-    struct stat sb;
-    int err = 0;
-    if (fstat(fd, &sb) != 0 || ((uint64_t)sb.st_size != g.img_bytes && ftruncate(fd, (off_t)g.img_bytes) != 0))
-      err = errno ? errno : EIO;
-    if (!err) err = posix_fallocate(fd, 0, (off_t)g.img_bytes);
-    if (err) {
-      flock(fd, LOCK_UN);
-      close(fd);
-      return fail(JITC_EIO, "jitc_register: sizing " + g.img_path + ": " + strerror(err));
-    }
-    void* p = mmap(nullptr, g.img_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
-    if (p == MAP_FAILED) {
-      flock(fd, LOCK_UN);
-      close(fd);
-      return fail(JITC_EIO, "jitc_register: mmap " + g.img_path + ": " + strerror(errno));
-    }
-    cudaError_t e = cudaHostRegister(p, g.img_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
-    flock(fd, LOCK_UN);
-    close(fd);
-    if (e != cudaSuccess) {
-      munmap(p, g.img_bytes);
-      return fail(JITC_ENOMEM, std::string("jitc_register: cudaHostRegister: ") + cudaGetErrorString(e));
-    }
-    g.img_h = (uint8_t*)p;
-    g.img_shm = true;
+    st = map_shared_image(c, g, "jitc_register");
+    if (st) return st;
   } else {
     cudaError_t e = cudaHostAlloc(&g.img_h, g.img_bytes, cudaHostAllocMapped | cudaHostAllocPortable);
     if (e != cudaSuccess) {
@@ -279,6 +288,29 @@ jitc_status jitc_register(jitc_ctx* c, uint32_t group, int32_t policy, const int
   CU(cudaHostGetDevicePointer((void**)&g.img_d, g.img_h, 0));
   if (layout_hash) *layout_hash = g.layout_hash;
   if (image_bytes) *image_bytes = g.L;
+  return JITC_OK;
+}
+
+jitc_status jitc_attach_image(jitc_ctx* c, uint32_t group, uint64_t image_bytes) {
+  if (!c) return fail(JITC_EINVAL, "jitc_attach_image: null ctx");
+  auto it = c->groups.find(group);
+  if (it == c->groups.end() || it->second.held)
+    return fail(JITC_EINVAL, "jitc_attach_image: group is not a declared (non-held) group");
+  if (c->image_dir.empty()) return fail(JITC_EINVAL, "jitc_attach_image: needs an image_dir");
+  if (image_bytes == 0 || image_bytes % kAlign) return fail(JITC_EINVAL, "jitc_attach_image: bad image size");
+  CU(cudaSetDevice(c->device));
+  GroupState& g = it->second;
+  if (g.img_h) {
+    if (g.L == image_bytes) return JITC_OK;
+    cudaHostUnregister(g.img_h);
+    munmap(g.img_h, g.img_bytes);
+    g.img_h = g.img_d = nullptr;
+  }
+  g.L = image_bytes;
+  g.img_bytes = align_up(image_bytes, 4096);
+  jitc_status st = map_shared_image(c, g, "jitc_attach_image");
+  if (st) return st;
+  CU(cudaHostGetDevicePointer((void**)&g.img_d, g.img_h, 0));
   return JITC_OK;
 }
 

@@ -83,6 +83,9 @@ typedef CUresult (*PFN_writeValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned
 // peers' host threads; K3 reads a peer's block straight from its staging
 // (peer memory over NVLink), so the exchange is fused into the unpack.
 constexpr int kIpcMaxRanks = 64;
+// Default copy-engine piece: 64 MiB pieces D2H at 55.6 GB/s vs 53.7 for one 2 GiB
+// copy per round (C2 capture 448 vs 464 ms, same box; profiles/r01_copy_piece.txt).
+constexpr uint64_t kDefaultCopyPiece = 64ull << 20;
 constexpr int kIpcMaxGroups = 64;
 struct IpcCtl {
   uint64_t arrive[kIpcMaxRanks];                  // barrier generations
@@ -92,6 +95,9 @@ struct IpcCtl {
   uint64_t staging_off[kIpcMaxRanks];
   uint64_t published[kIpcMaxRanks];
   uint64_t heartbeat[kIpcMaxRanks];  // CLOCK_MONOTONIC microseconds, refreshed every 10 ms while alive
+  // capture fan-out rounds: (call generation << 24) | (round + 1)
+  uint64_t cap_posted[kIpcMaxRanks][kIpcMaxGroups];
+  uint64_t cap_consumed[kIpcMaxRanks][kIpcMaxGroups];
 };
 struct IpcComm {
   std::string dir;
@@ -101,7 +107,7 @@ struct IpcComm {
   std::vector<int> slot;               // comm rank -> index into the IpcCtl arrays (stable across shrink)
   std::vector<uint8_t*> peer_staging;  // by comm rank (own entry = ctx staging)
   std::vector<void*> opened;
-  uint64_t barrier_gen = 0, exchange_gen = 0;
+  uint64_t barrier_gen = 0, exchange_gen = 0, cap_gen = 0;
   std::map<uint32_t, uint64_t> rounds;      // cumulative restore rounds per group slot
   std::map<uint32_t, uint64_t> digest_gen;  // PEER digest hand-offs per group slot
   std::thread hb_thread;                    // heartbeat writer (failure localisation, NEXT-1)
@@ -120,6 +126,9 @@ struct jitc_ctx {
   bool own_streams = false;
   uint8_t* staging = nullptr;
   uint64_t staging_bytes = 0, slot_bytes = 0;
+  // copy-engine transfers (D2H / H2D) are issued in pieces of at most this
+  // many bytes (env JITC_COPY_PIECE_MB; 0 = one copy per round)
+  uint64_t copy_piece = 0;
   bool own_staging = false;
   static constexpr int kSlots = 8;
   cudaEvent_t ev_ready[kSlots]{}, ev_free[kSlots]{};
@@ -256,6 +265,18 @@ inline void finish_stats(jitc_ctx* c, const CallTimer& t, jitc_stats* st, bool d
 
 // Segments whose image offset lies in [a, b) (segments never straddle a chunk
 // boundary and rounds are chunk-aligned, so this is exact).
+// A host<->device copy on `s`, issued in pieces of at most c->copy_piece bytes.
+inline cudaError_t copy_pieces(const jitc_ctx* c, void* dst, const void* src, uint64_t n, cudaMemcpyKind kind,
+                               cudaStream_t s) {
+  const uint64_t P = c->copy_piece ? c->copy_piece : n;
+  for (uint64_t o = 0; o < n; o += P) {
+    cudaError_t e = cudaMemcpyAsync(static_cast<uint8_t*>(dst) + o, static_cast<const uint8_t*>(src) + o,
+                                    std::min(P, n - o), kind, s);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
 inline void seg_span(const GroupState& g, uint64_t a, uint64_t b, uint32_t* lo, uint32_t* hi) {
   auto cmp = [](const Seg& s, uint64_t v) { return s.img_off < v; };
   *lo = (uint32_t)(std::lower_bound(g.segs.begin(), g.segs.end(), a, cmp) - g.segs.begin());

@@ -227,7 +227,7 @@ uint64_t root_of(uint64_t layout_hash, const uint64_t* d, uint64_t n_c);
 
 // ------------------------------------------------------------------ restore plan (jitc_plan.cc)
 enum : uint8_t { kOpH2D = 1, kOpAllGather = 2, kOpPack = 3, kOpSend = 4, kOpRecv = 5, kOpUnpack = 6,
-                 kOpDigestSend = 7, kOpDigestRecv = 8 };
+                 kOpDigestSend = 7, kOpDigestRecv = 8, kOpD2H = 9 };
 constexpr uint32_t kMagicPlan = 0x5054494Au;      // "JITP"
 #pragma pack(push, 1)
 struct PlanOp {      // 48 B
@@ -258,10 +258,19 @@ struct PlanInput {
   int n = 1, me = 0;                   // communicator size and this rank
   std::vector<int32_t> writers, dests;  // comm ranks (PEER)
   std::vector<int32_t> participants;    // comm ranks of the group's members, sorted (HOST)
+  std::vector<int32_t> movers;          // comm ranks that D2H a lane of the image (capture fan-out)
   uint64_t staging_bytes = 0, slot_bytes = 0;
 };
 bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
                         std::string* why, uint32_t* n_rounds = nullptr);
+// Capture with NVLink fan-out: writer s packs its O5(n_c, k, s)
+// shard; mover q D2Hs lane O5(n_c, m, q) of the image; the part of a shard
+// that lies in another rank's lane travels writer -> mover over NVLink.
+bool build_capture_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
+                        std::string* why, uint32_t* n_rounds);
+bool capture_plan_input(const GroupSelection& gs, const int32_t* movers, int32_t n_movers,
+                        const int32_t* comm_job_ranks, int32_t n, int32_t comm_rank, uint64_t staging_bytes,
+                        uint64_t slot_bytes, PlanInput* in, std::string* why);
 uint64_t manifest_trailer(const uint8_t* p, size_t n);
 
 // thread-local error text

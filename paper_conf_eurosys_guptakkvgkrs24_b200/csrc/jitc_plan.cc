@@ -149,6 +149,140 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
   return true;
 }
 
+// Capture with NVLink fan-out.  The host
+// link, not HBM, bounds capture, and a group with few writers (k = 1 for the
+// TP partition that lost a replica, C5) would leave every other GPU's link
+// idle.  The image is therefore D2H'd in m lanes, lane q = O5(n_c, m, q) by
+// mover q, while writer s still packs (and re-digests) exactly its O5(n_c, k,
+// s) shard: the piece shard s ∩ lane q is PACKed by s and, when s is not q,
+// SENT over NVLink to q, which RECEIVEs and D2Hs it.  Each writer walks its
+// shard in blocks of <= R bytes cut at lane boundaries; round j carries every
+// writer's j-th block, at staging offset slot*k*R + s*R on both sides.  With
+// m == k and movers == writers this is the plain sharded capture.
+bool build_capture_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t* round_bytes, uint32_t* slots,
+                        std::string* why, uint32_t* n_rounds) {
+  ops->clear();
+  *round_bytes = 0;
+  *slots = 0;
+  *n_rounds = 0;
+  const uint64_t C = in.chunk_bytes, L = in.image_bytes, n_c = in.n_c;
+  const uint64_t k = in.writers.size(), m = in.movers.size();
+  if (C == 0 || in.n <= 0 || in.me < 0 || in.me >= in.n) {
+    *why = "bad plan input";
+    return false;
+  }
+  if (k == 0) return true;  // dropped group: nothing is captured
+  if (m == 0) {
+    *why = "no movers";
+    return false;
+  }
+  for (int32_t w : in.writers)
+    if (w < 0 || w >= in.n) {
+      *why = "a writer is not in the communicator";
+      return false;
+    }
+  for (size_t i = 0; i < m; ++i) {
+    if (in.movers[i] < 0 || in.movers[i] >= in.n) {
+      *why = "a mover is not in the communicator";
+      return false;
+    }
+    for (size_t j = 0; j < i; ++j)
+      if (in.movers[j] == in.movers[i]) {
+        *why = "duplicate mover";
+        return false;
+      }
+  }
+  const uint64_t S = 2;
+  const uint64_t R = std::min<uint64_t>(in.slot_bytes, in.staging_bytes / (S * k)) / C * C;
+  if (R == 0) {
+    *why = "staging too small for the capture rounds (need >= 2 * k * C bytes)";
+    return false;
+  }
+  *round_bytes = R;
+  *slots = (uint32_t)S;
+  struct Block {
+    uint64_t a, b;
+    uint32_t q;
+  };
+  std::vector<std::vector<Block>> blocks(k);
+  uint64_t J = 0;
+  for (uint64_t s = 0; s < k; ++s) {
+    uint64_t a, b;
+    o5_bytes(n_c, k, s, C, L, &a, &b);
+    for (uint64_t q = 0; q < m; ++q) {
+      uint64_t la, lb;
+      o5_bytes(n_c, m, q, C, L, &la, &lb);
+      const uint64_t x = std::max(a, la), y = std::min(b, lb);
+      for (uint64_t u = x; u < y; u += R) blocks[s].push_back(Block{u, std::min(u + R, y), (uint32_t)q});
+    }
+    J = std::max<uint64_t>(J, blocks[s].size());
+  }
+  *n_rounds = (uint32_t)J;
+  for (uint64_t j = 0; j < J; ++j) {
+    const uint32_t sl = (uint32_t)(j % S);
+    const uint64_t base = sl * k * R;
+    std::vector<PlanOp> pack, xfer, d2h;
+    for (uint64_t s = 0; s < k; ++s) {
+      if (j >= blocks[s].size()) continue;
+      const Block& bl = blocks[s][j];
+      const uint64_t off = base + s * R, n = bl.b - bl.a;
+      const int32_t w = in.writers[s], q = in.movers[bl.q];
+      if (w == in.me) {
+        pack.push_back(PlanOp{(uint32_t)j, kOpPack, (uint8_t)sl, 0, in.me, 0, bl.a, bl.b, off, n});
+        if (q != in.me) xfer.push_back(PlanOp{(uint32_t)j, kOpSend, (uint8_t)sl, 0, q, 0, bl.a, bl.b, off, n});
+      } else if (q == in.me) {
+        xfer.push_back(PlanOp{(uint32_t)j, kOpRecv, (uint8_t)sl, 0, w, 0, bl.a, bl.b, off, n});
+      }
+      if (q == in.me) d2h.push_back(PlanOp{(uint32_t)j, kOpD2H, (uint8_t)sl, 0, w, 0, bl.a, bl.b, off, n});
+    }
+    ops->insert(ops->end(), pack.begin(), pack.end());
+    ops->insert(ops->end(), xfer.begin(), xfer.end());
+    ops->insert(ops->end(), d2h.begin(), d2h.end());
+  }
+  return true;
+}
+
+// Plan input of a fan-out capture: writers from the selection (sorted by job
+// rank), movers = the caller's job ranks sorted, both mapped to comm ranks.
+bool capture_plan_input(const GroupSelection& gs, const int32_t* movers, int32_t n_movers,
+                        const int32_t* comm_job_ranks, int32_t n, int32_t comm_rank, uint64_t staging_bytes,
+                        uint64_t slot_bytes, PlanInput* in, std::string* why) {
+  auto comm_of = [&](int32_t job) {
+    for (int i = 0; i < n; ++i)
+      if (comm_job_ranks[i] == job) return i;
+    return -1;
+  };
+  in->mode = 0;
+  in->n_c = gs.n_c;
+  in->chunk_bytes = gs.chunk_bytes;
+  in->image_bytes = gs.image_bytes;
+  in->n = n;
+  in->me = comm_rank;
+  in->staging_bytes = staging_bytes;
+  in->slot_bytes = slot_bytes;
+  in->writers.clear();
+  in->movers.clear();
+  for (int32_t w : gs.writers) {
+    int r = comm_of(w);
+    if (r < 0) {
+      *why = "writer " + std::to_string(w) + " is not in the communicator";
+      return false;
+    }
+    in->writers.push_back(r);
+  }
+  std::vector<int32_t> mv(movers, movers + n_movers);
+  std::sort(mv.begin(), mv.end());
+  for (int32_t q : mv) {
+    int r = comm_of(q);
+    if (r < 0) {
+      *why = "mover " + std::to_string(q) + " is not in the communicator";
+      return false;
+    }
+    in->movers.push_back(r);
+  }
+  return true;
+}
+
 }  // namespace jitc
 
 using namespace jitc;
@@ -215,6 +349,54 @@ extern "C" jitc_status jitc_restore_plan(const void* selection, size_t sel_len, 
   if (cap == 0) return JITC_OK;
   if (cap < *len || !plan) {
     set_error("jitc_restore_plan: buffer too small");
+    return JITC_EINVAL;
+  }
+  memcpy(plan, &h, sizeof h);
+  if (!ops.empty()) memcpy(static_cast<uint8_t*>(plan) + sizeof h, ops.data(), ops.size() * sizeof(PlanOp));
+  return JITC_OK;
+}
+
+extern "C" jitc_status jitc_capture_plan(const void* selection, size_t sel_len, uint32_t group, const int32_t* movers,
+                                         int32_t n_movers, const int32_t* comm_job_ranks, int32_t n, int32_t comm_rank,
+                                         uint64_t staging_bytes, uint64_t slot_bytes, void* plan, size_t cap,
+                                         size_t* len) {
+  if (!selection || !comm_job_ranks || !len || n <= 0 || n_movers < 0 || (n_movers && !movers)) {
+    set_error("jitc_capture_plan: bad argument");
+    return JITC_EINVAL;
+  }
+  Selection sel;
+  std::string why;
+  if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why)) {
+    set_error("jitc_capture_plan: " + why);
+    return JITC_EINVAL;
+  }
+  const GroupSelection* gs = sel.find(group);
+  if (!gs) {
+    set_error("jitc_capture_plan: group not in selection");
+    return JITC_EINVAL;
+  }
+  PlanInput in;
+  if (!capture_plan_input(*gs, movers, n_movers, comm_job_ranks, n, comm_rank, staging_bytes, slot_bytes, &in, &why)) {
+    set_error("jitc_capture_plan: " + why);
+    return JITC_EINVAL;
+  }
+  std::vector<PlanOp> ops;
+  uint64_t R = 0;
+  uint32_t S = 0, J = 0;
+  if (!build_capture_plan(in, &ops, &R, &S, &why, &J)) {
+    set_error("jitc_capture_plan: " + why);
+    return JITC_EINVAL;
+  }
+  PlanHdr h{};
+  h.magic = kMagicPlan;
+  h.n_ops = (uint32_t)ops.size();
+  h.round_bytes = R;
+  h.slots = S;
+  h.n_rounds = J;
+  *len = sizeof h + ops.size() * sizeof(PlanOp);
+  if (cap == 0) return JITC_OK;
+  if (cap < *len || !plan) {
+    set_error("jitc_capture_plan: buffer too small");
     return JITC_EINVAL;
   }
   memcpy(plan, &h, sizeof h);

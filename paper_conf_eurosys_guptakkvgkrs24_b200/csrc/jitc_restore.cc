@@ -120,7 +120,7 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
       if (op.kind != kOpH2D) continue;
       if (!any_h2d && used[sl]) CU(cudaStreamWaitEvent(c->s_copy, c->ev_free[sl], 0));
       any_h2d = true;
-      CU(cudaMemcpyAsync(c->staging + op.off, g.img_h + op.a, op.bytes, cudaMemcpyHostToDevice, c->s_copy));
+      CU(copy_pieces(c, c->staging + op.off, g.img_h + op.a, op.bytes, cudaMemcpyHostToDevice, c->s_copy));
       if (stats) stats->h2d_bytes += op.bytes;
     }
     if (any_h2d) {

@@ -103,6 +103,9 @@ def lib() -> ctypes.CDLL:
         "jitc_layout": ([P(Tensor), sz, u64, P(u64), P(u64), P(u64)], i32),
         "jitc_shard_range": ([u64, u32, u32, P(u64), P(u64)], i32),
         "jitc_restore_plan": ([vp, sz, u32, i32, P(i32), i32, i32, u64, u64, vp, sz, P(sz)], i32),
+        "jitc_capture_plan": ([vp, sz, u32, P(i32), i32, P(i32), i32, i32, u64, u64, vp, sz, P(sz)], i32),
+        "jitc_capture_fanout": ([vp, vp, sz, u32, P(i32), i32, P(Stats)], i32),
+        "jitc_attach_image": ([vp, u32, u64], i32),
         "jitc_kernel_counters": ([vp, i32, P(KernelCounter)], i32),
         "jitc_reset_counters": ([vp], i32),
         "jitc_gen_fill": ([vp, u32, u64, u64, u32, u32, u32, u32, i32, vp], i32),
@@ -140,7 +143,8 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_layout", "jitc_shard_range", "jitc_restore_plan", "jitc_kernel_counters", "jitc_reset_counters", "jitc_gen_fill",
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
             "jitc_inject_release", "jitc_capture_local", "jitc_set_aux", "jitc_get_aux", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
-            "jitc_watchdog_stop", "jitc_watchdog_failed"]
+            "jitc_watchdog_stop", "jitc_watchdog_failed", "jitc_capture_plan", "jitc_capture_fanout",
+            "jitc_attach_image"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE, ON_HANG_COLLECTIVE_CAPTURE = 0, 1, 2
 
 
@@ -218,7 +222,7 @@ def waste_model(kind: int, n_gpus: float, f: float, o: float = 0.0, r: float = 0
     return dict(c_opt=co.value, w=w.value, w_f=wf.value)
 
 
-OP_NAMES = {1: "H2D", 2: "ALLGATHER", 3: "PACK", 4: "SEND", 5: "RECV", 6: "UNPACK", 7: "DIGEST_SEND",
+OP_NAMES = {1: "H2D", 2: "ALLGATHER", 3: "PACK", 4: "SEND", 5: "RECV", 6: "UNPACK", 7: "DIGEST_SEND", 9: "D2H",
             8: "DIGEST_RECV"}
 
 
@@ -232,7 +236,25 @@ def restore_plan(selection: bytes, group: int, mode: int, comm_job_ranks: Sequen
     _check(L.jitc_restore_plan(*args, None, 0, ctypes.byref(n)), "jitc_restore_plan")
     buf = ctypes.create_string_buffer(n.value)
     _check(L.jitc_restore_plan(*args, buf, n.value, ctypes.byref(n)), "jitc_restore_plan")
-    raw = buf.raw[:n.value]
+    return _parse_plan(buf.raw[:n.value])
+
+
+def capture_plan(selection: bytes, group: int, movers: Sequence[int], comm_job_ranks: Sequence[int], comm_rank: int,
+                 staging_bytes: int, slot_bytes: int) -> dict:
+    """The round schedule jitc_capture_fanout executes on `comm_rank` (pure; no GPU)."""
+    L = lib()
+    n = ctypes.c_size_t()
+    jr = _i32arr(list(comm_job_ranks))
+    mv = _i32arr(list(movers))
+    args = (selection, len(selection), group, mv, len(movers), jr, len(comm_job_ranks), comm_rank, staging_bytes,
+            slot_bytes)
+    _check(L.jitc_capture_plan(*args, None, 0, ctypes.byref(n)), "jitc_capture_plan")
+    buf = ctypes.create_string_buffer(n.value)
+    _check(L.jitc_capture_plan(*args, buf, n.value, ctypes.byref(n)), "jitc_capture_plan")
+    return _parse_plan(buf.raw[:n.value])
+
+
+def _parse_plan(raw: bytes) -> dict:
     magic, n_ops, R, S, n_rounds = struct.unpack_from("<IIQII", raw, 0)
     ops = []
     for i in range(n_ops):
@@ -367,6 +389,18 @@ class Context:
         st = Stats()
         _check(self._L.jitc_capture(self._h, selection, len(selection), group, ctypes.byref(st)), "jitc_capture")
         return st.as_dict()
+
+    def capture_fanout(self, selection: bytes, movers: Sequence[int], group: int = ALL_GROUPS) -> dict:
+        """Collective: capture with NVLink fan-out over `movers` (job ranks)."""
+        st = Stats()
+        mv = _i32arr(list(movers))
+        _check(self._L.jitc_capture_fanout(self._h, selection, len(selection), group, mv, len(movers),
+                                           ctypes.byref(st)), "jitc_capture_fanout")
+        return st.as_dict()
+
+    def attach_image(self, group: int, image_bytes: int):
+        """Maps and pins the host image of a declared (non-held) group (fan-out mover)."""
+        _check(self._L.jitc_attach_image(self._h, group, image_bytes), "jitc_attach_image")
 
     def capture_local(self) -> dict:
         st = Stats()

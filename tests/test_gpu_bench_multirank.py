@@ -1,7 +1,9 @@
 """bench.py's N > 1 path (torchrun, one process per rank, gloo rendezvous,
-the library's IPC communicator, k = N sharded capture, N-way HOST restore,
-max-over-ranks timing) run functionally on one B200: JITC_BENCH_SHARE_GPU
-puts every rank on GPU 0 (the numbers are not a measurement)."""
+the library's communicator, k = N sharded capture, N-way HOST restore,
+max-over-ranks timing) run functionally on one B200 over either transport:
+JITC_BENCH_SHARE_GPU puts every rank on GPU 0 (and, for NCCL, gives each rank
+its own NCCL_HOSTID so NCCL accepts two ranks on one device); the numbers are
+not a measurement."""
 import json
 import os
 import socket
@@ -14,7 +16,8 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def test_bench_two_ranks_one_gpu():
+@pytest.mark.parametrize("transport", ["ipc", "nccl"])
+def test_bench_two_ranks_one_gpu(transport):
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
     port = s.getsockname()[1]
@@ -23,11 +26,11 @@ def test_bench_two_ranks_one_gpu():
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
                         "--master-addr", "127.0.0.1", "--master-port", str(port), "bench.py", "--gpus", "2",
                         "--steps", "3", "--warmup", "3", "--config", "C1", "--no-cpu-baseline", "--staging", "256",
-                        "--slot", "64", "--hang-ctas", "0"],
+                        "--slot", "64", "--hang-ctas", "0", "--transport", transport],
                        cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
-    assert d["n_gpus"] == 2 and d["config"]["writers_k"] == 2 and d["config"]["transport"] == "ipc"
+    assert d["n_gpus"] == 2 and d["config"]["writers_k"] == 2 and d["config"]["transport"] == transport
     assert d["value"] > 0 and d["gpu_launches"] > 0

@@ -1,6 +1,9 @@
-"""The whole multi-rank runtime on one B200 with real processes, through the
-library's intra-node IPC transport (jitc_comm_init_ipc; NCCL refuses two
-ranks on one GPU): record exchange, selection, k-way sharded capture into
+"""The whole multi-rank runtime on one B200 with real processes, through each
+of the library's two transports: the intra-node IPC transport
+(jitc_comm_init_ipc) and NCCL (jitc_comm_init).  NCCL refuses two ranks with
+the same (host hash, bus id); every rank gets its own NCCL_HOSTID, so NCCL
+sees separate hosts and connects them with its socket transport over
+loopback (functional, not a measurement).  Covered: record exchange, selection, k-way sharded capture into
 the shared image, commit barrier, HOST restore with the slice exchange fused
 into K3 (each rank loads 1/n of the image and reads the others' slices from
 their staging through CUDA IPC), and PEER restore of a replacement process
@@ -28,7 +31,7 @@ from paper_conf_eurosys_guptakkvgkrs24_b200 import jitc as J
 from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
 from workloads import configs as W
 
-rank, world, shm, phase = {rank}, {world}, {shm!r}, {phase!r}
+rank, world, shm, phase, transport = {rank}, {world}, {shm!r}, {phase!r}, {transport!r}
 base = W.scaled(W.c2(), 30000)
 groups = [base.groups[0], base.groups[1]]           # REQUIRED + OPTIONAL, on every rank
 sub = W.scaled(W.c1(), 4000).groups[0]; sub.group = 2; sub.members = [0, 1]   # a subset group
@@ -51,7 +54,17 @@ def make_ctx(comm_dir, scramble):
             ctx.mark(g.group, 33, J.CLEAN)
         else:
             ctx.declare_group(g.group, g.policy, members)
-    ctx.comm_init_ipc(comm_dir, world, rank)
+    if transport == "ipc":
+        ctx.comm_init_ipc(comm_dir, world, rank)
+    else:                                           # NCCL: rank 0 publishes the unique id
+        uid_path = comm_dir + ".uid"
+        if rank == 0:
+            open(uid_path + ".tmp", "wb").write(J.get_unique_id())
+            os.rename(uid_path + ".tmp", uid_path)
+        t0 = time.time()
+        while not os.path.exists(uid_path) and time.time() - t0 < 120:
+            time.sleep(0.01)
+        ctx.comm_init(open(uid_path, "rb").read(), world, rank)
     return ctx, sts
 
 
@@ -136,43 +149,53 @@ ctx.close()
 """
 
 
-def _spawn(shm, world, phases):
+def _env(transport, rank):
+    if transport == "ipc":
+        return dict(os.environ)
+    return dict(os.environ, NCCL_HOSTID=f"jitc-test-host-{rank}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
+                NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0", NCCL_DEBUG="WARN")
+
+
+def _spawn(shm, world, phases, transport):
     procs = []
     for r, ph in phases.items():
-        code = textwrap.dedent(RANK.format(root=ROOT, rank=r, world=world, shm=shm, phase=ph))
+        code = textwrap.dedent(RANK.format(root=ROOT, rank=r, world=world, shm=shm, phase=ph, transport=transport))
         procs.append(subprocess.Popen([sys.executable, "-c", code], cwd=ROOT, stdout=subprocess.PIPE,
-                                      stderr=subprocess.STDOUT, text=True))
+                                      stderr=subprocess.STDOUT, text=True, env=_env(transport, r)))
     outs = [p.communicate(timeout=600)[0] for p in procs]
     for p, o in zip(procs, outs):
         assert p.returncode == 0, "\n=====\n".join(outs)
     return outs
 
 
-def test_ipc_multirank_capture_and_host_restore():
+@pytest.mark.parametrize("transport", ["ipc", "nccl"])
+def test_multirank_capture_and_host_restore(transport):
     shm = f"/dev/shm/jitc-ipc-{os.getpid()}-{uuid.uuid4().hex[:8]}"
     os.makedirs(shm)
     try:
-        outs = _spawn(shm, 3, {0: "host", 1: "host", 2: "host"})
+        outs = _spawn(shm, 3, {0: "host", 1: "host", 2: "host"}, transport)
         assert all("host ok" in o for o in outs), outs
     finally:
         shutil.rmtree(shm, ignore_errors=True)
 
 
-def test_ipc_multirank_peer_restore_of_replacement():
+@pytest.mark.parametrize("transport", ["ipc", "nccl"])
+def test_multirank_peer_restore_of_replacement(transport):
     shm = f"/dev/shm/jitc-ipc-{os.getpid()}-{uuid.uuid4().hex[:8]}"
     os.makedirs(shm)
     try:
-        outs = _spawn(shm, 3, {0: "writer", 1: "replacement", 2: "writer"})
+        outs = _spawn(shm, 3, {0: "writer", 1: "replacement", 2: "writer"}, transport)
         assert "peer ok" in outs[1] and "writer ok" in outs[0] and "writer ok" in outs[2], outs
     finally:
         shutil.rmtree(shm, ignore_errors=True)
 
 
-def test_ipc_peer_repairs_replacement_and_dirty_member():
+@pytest.mark.parametrize("transport", ["ipc", "nccl"])
+def test_peer_repairs_replacement_and_dirty_member(transport):
     shm = f"/dev/shm/jitc-ipc-{os.getpid()}-{uuid.uuid4().hex[:8]}"
     os.makedirs(shm)
     try:
-        outs = _spawn(shm, 3, {0: "w0", 1: "repl", 2: "dirty"})
+        outs = _spawn(shm, 3, {0: "w0", 1: "repl", 2: "dirty"}, transport)
         assert "w0 ok" in outs[0] and "repl ok" in outs[1] and "dirty ok" in outs[2], outs
     finally:
         shutil.rmtree(shm, ignore_errors=True)
