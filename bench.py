@@ -88,6 +88,83 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(self.rows)}
 
 
+def calibrate_links(device: int, world: int, nccl_group=None, host_gib: int = 2):
+    """In-run link calibration, untimed, before the
+    timed region: B_d2h / B_h2d with every rank copying at once (64 MiB
+    cudaMemcpyAsync pieces of pinned memory, best of 3), B_hbm from a 4 GiB
+    device-to-device copy (read + write bytes), B_nvl from a 256 MiB-per-rank
+    NCCL all-gather (bus bandwidth (n-1)/n * total / t) when an NCCL group is
+    given.  Returns GB/s (per rank for the host link)."""
+    import torch
+    import torch.distributed as dist
+    n = host_gib << 30
+    piece = 64 << 20
+    h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(n, dtype=torch.uint8, device=f"cuda:{device}")
+    s = torch.cuda.Stream(device)
+    out = {}
+
+    def timed(fn, reps=3):
+        best = None
+        for _ in range(reps):
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(s):
+                e0.record(s)
+                fn()
+                e1.record(s)
+            e1.synchronize()
+            t = e0.elapsed_time(e1) * 1e-3
+            best = t if best is None else min(best, t)
+        return best
+
+    def d2h():
+        for o in range(0, n, piece):
+            h[o:o + piece].copy_(d[o:o + piece], non_blocking=True)
+
+    def h2d():
+        for o in range(0, n, piece):
+            d[o:o + piece].copy_(h[o:o + piece], non_blocking=True)
+
+    out["d2h_GBps"] = round(n / timed(d2h) / 1e9, 2)
+    out["h2d_GBps"] = round(n / timed(h2d) / 1e9, 2)
+    del h
+    a = torch.empty(4 << 30, dtype=torch.uint8, device=f"cuda:{device}")
+    b = torch.empty_like(a)
+    out["hbm_copy_GBps"] = round(2 * a.numel() / timed(lambda: b.copy_(a)) / 1e9, 1)
+    del a, b, d
+    if nccl_group is not None and world > 1:
+        blk = torch.empty(256 << 20, dtype=torch.uint8, device=f"cuda:{device}")
+        allb = torch.empty(world * blk.numel(), dtype=torch.uint8, device=f"cuda:{device}")
+        t = timed(lambda: dist.all_gather_into_tensor(allb, blk, group=nccl_group))
+        out["nvl_allgather_busbw_GBps"] = round((world - 1) * blk.numel() / t / 1e9, 1)
+    torch.cuda.empty_cache()
+    out["how"] = (f"{host_gib} GiB pinned, 64 MiB pieces, all {world} rank(s) at once, best of 3; "
+                  "HBM: 4 GiB D2D copy (read+write)")
+    return out
+
+
+def host_link_roofline(L_total, world, capture_ms, restore_ms, links):
+    """Capture / restore GB/s per rank against the host link: nominal PCIe
+    Gen5 x16, the pool's probe (profiles/r01_pcie_probe.txt) and, when run,
+    this run's own calibration (calibrate_links, all ranks at once)."""
+    cap = L_total / world / (capture_ms * 1e-3) / 1e9
+    res = L_total / world / (restore_ms * 1e-3) / 1e9
+    out = {"capture_GBps_per_rank": round(cap, 2), "restore_GBps_per_rank": round(res, 2),
+           "nominal_GBps": HOST_LINK_NOMINAL, "probe_GBps": HOST_LINK_MEASURED,
+           "capture_frac_nominal": round(cap / HOST_LINK_NOMINAL, 3),
+           "restore_frac_nominal": round(res / HOST_LINK_NOMINAL, 3),
+           "capture_frac_probe": round(cap / HOST_LINK_MEASURED["d2h"], 3),
+           "restore_frac_probe": round(res / HOST_LINK_MEASURED["h2d"], 3)}
+    if links:
+        out["calibrated"] = links
+        out["capture_frac_calibrated"] = round(cap / links["d2h_GBps"], 3)
+        out["restore_frac_calibrated"] = round(res / links["h2d_GBps"], 3)
+    return out
+
+
 # ---------------------------------------------------------------------- reference arm / cpu baseline
 def oracle_sample(cfg_name: str, sample_bytes: int):
     """Generates a bounded, contiguous prefix of the configuration's REQUIRED
@@ -221,6 +298,10 @@ def run_jitc(args):
     comm_init_ms = (time.perf_counter() - t_comm) * 1e3
     torch.cuda.synchronize()
     setup_s = time.perf_counter() - t_setup
+    nccl_group = None
+    if world > 1 and not os.environ.get("JITC_BENCH_SHARE_GPU"):
+        nccl_group = dist.new_group(backend="nccl")
+    links = calibrate_links(local, world, nccl_group) if not args.no_calibrate else None
 
     healthy = list(range(world))
     per = {"fingerprint": [], "select": [], "capture": [], "commit": [], "restore": [], "verify": []}
@@ -305,6 +386,9 @@ def run_jitc(args):
     ms_per_launch = c["ms"] / max(c["launches"], 1)
     peak, peak_src = _peaks()
     achieved = bytes_per_launch / (ms_per_launch * 1e-3) / 1e9 if ms_per_launch > 0 else None
+    # diagnostic: the same launches timed inside the kernel (first CTA start -> last CTA end, %globaltimer)
+    span_per_launch = c.get("span_ms", 0.0) / max(c["launches"], 1)
+    achieved_span = bytes_per_launch / (span_per_launch * 1e-3) / 1e9 if span_per_launch > 0 else None
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
@@ -333,16 +417,17 @@ def run_jitc(args):
             "phases_ms_median": med,
             "capture_GBps": round(L_total / world / (cap_ms * 1e-3) / 1e9, 3),
             "restore_GBps": round(L_total / (res_ms * 1e-3) / 1e9, 3),
-            "host_link_roofline": {"nominal_GBps": HOST_LINK_NOMINAL, "measured_GBps": HOST_LINK_MEASURED,
-                                   "capture_frac_nominal": round(L_total / world / (med["capture"] * 1e-3) / 1e9 / HOST_LINK_NOMINAL, 3),
-                                   "restore_frac_nominal": round(L_total / world / (res_ms * 1e-3) / 1e9 / HOST_LINK_NOMINAL, 3),
-                                   "capture_frac_measured": round(L_total / world / (med["capture"] * 1e-3) / 1e9 / HOST_LINK_MEASURED["d2h"], 3),
-                                   "restore_frac_measured": round(L_total / world / (res_ms * 1e-3) / 1e9 / HOST_LINK_MEASURED["h2d"], 3)},
+            "host_link_roofline": host_link_roofline(L_total, world, med["capture"], res_ms, links),
             "roofline": {"kernel": kinds[dom], "bound": "hbm", "achieved": round(achieved, 1) if achieved else None,
                          "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
                          "traffic": traffic, "peak_source": peak_src,
                          "bytes_per_launch": bytes_per_launch, "ms_per_launch": round(ms_per_launch, 4),
-                         "launches": c["launches"]},
+                         "launches": c["launches"],
+                         "kernel_span": {"ms_per_launch": round(span_per_launch, 4),
+                                         "achieved": round(achieved_span, 1) if achieved_span else None,
+                                         "frac": round(achieved_span / peak, 4) if achieved_span else None,
+                                         "how": "diagnostic: %globaltimer first-CTA-start to last-CTA-end per launch; "
+                                                "`achieved` above is the CUDA-event figure"}},
             "kernels": {kinds[k]: {"launches": kc[k]["launches"], "ms": round(kc[k]["ms"], 3),
                                    "GBps": round((1 if k == J.K_DIGEST else 2) * kc[k]["bytes"] / (kc[k]["ms"] * 1e-3) / 1e9, 1)
                                    if kc[k]["ms"] else None} for k in kinds},
@@ -372,10 +457,13 @@ def main():
     ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3"])
     ap.add_argument("--impl", default="jitc", choices=["jitc", "reference"])
     ap.add_argument("--staging", type=int, default=8192, help="MiB of device staging")
-    ap.add_argument("--slot", type=int, default=2048, help="MiB per pipeline round")
+    ap.add_argument("--slot", type=int, default=4096,
+                    help="MiB per pipeline round (4 GiB: the ~45 us per-launch cost of running next to a copy-engine "
+                         "transfer is amortised over 8.6 GB of K2/K3 traffic; profiles/r01_slot_size.txt)")
     ap.add_argument("--zero-copy", action="store_true")
     ap.add_argument("--image-dir", default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-calibrate", action="store_true", help="skip the in-run host-link / HBM / NVLink calibration")
     ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],
                     help="N > 1 communicator: intra-node CUDA IPC (default; tested on B200 with real processes) or NCCL")

@@ -141,6 +141,8 @@ typedef struct {
     uint64_t launches;
     uint64_t bytes;            /* algorithmic image bytes processed                            */
     double ms;                 /* sum of CUDA-event launch durations (JITC_F_TIME_KERNELS)     */
+    double span_ms;            /* sum of in-kernel spans, first CTA start -> last CTA end
+                                  (%globaltimer; diagnostic, JITC_F_TIME_KERNELS)              */
 } jitc_kernel_counter;
 
 /* ---- lifecycle --------------------------------------------------------- */

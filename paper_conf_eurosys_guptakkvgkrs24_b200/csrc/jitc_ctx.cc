@@ -91,6 +91,9 @@ jitc_status jitc_create(const jitc_config* cfg, jitc_ctx** out) {
   if (c->cfg.flags & JITC_F_TIME_KERNELS) {
     c->kev.resize(2 * 2048);
     for (auto& ev : c->kev) CU(cudaEventCreate(&ev));
+    CU(cudaMalloc(&c->d_span, c->kev.size() * sizeof(unsigned long long)));
+    CU(cudaMemset(c->d_span, 0, c->kev.size() * sizeof(unsigned long long)));
+    c->h_span.assign(c->kev.size(), 0);
     c->kev_kind.resize(2048);
     c->kev_bytes.resize(2048);
   }
@@ -135,6 +138,7 @@ void jitc_destroy(jitc_ctx* c) {
   if (c->h_small) cudaFreeHost(c->h_small);
   if (c->d_small) cudaFree(c->d_small);
   if (c->d_work) cudaFree(c->d_work);
+  if (c->d_span) cudaFree(c->d_span);
   if (c->own_staging && c->staging) cudaFree(c->staging);
   if (c->own_streams) {
     cudaStreamDestroy(c->s_comp);

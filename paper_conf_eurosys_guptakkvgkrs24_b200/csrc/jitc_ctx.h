@@ -134,6 +134,8 @@ struct jitc_ctx {
   cudaEvent_t ev_ready[kSlots]{}, ev_free[kSlots]{};
   cudaEvent_t ev_t0 = nullptr, ev_t1 = nullptr, ev_join = nullptr;
   std::vector<cudaEvent_t> kev;  // kernel timing pairs
+  unsigned long long* d_span = nullptr;  // per timed launch: {~first CTA start, last CTA end} (%globaltimer)
+  std::vector<unsigned long long> h_span;
   std::vector<int> kev_kind;
   std::vector<uint64_t> kev_bytes;
   size_t kev_used = 0;
@@ -212,6 +214,7 @@ struct CallTimer {
     c->launches_in_call = 0;
     c->kernel_ms_in_call = 0;
     c->kev_used = 0;
+    if (c->d_span) cudaMemsetAsync(c->d_span, 0, c->kev.size() * sizeof(unsigned long long), c->s_comp);
   }
 };
 
@@ -226,7 +229,8 @@ inline jitc_status run_segments(jitc_ctx* c, GroupState& g, int mode, const Laun
                          uint64_t bytes, const uint64_t* remote = nullptr) {
   bool timed = (c->cfg.flags & JITC_F_TIME_KERNELS) && c->kev_used + 2 <= c->kev.size();
   if (timed) CU(cudaEventRecord(c->kev[c->kev_used], c->s_comp));
-  CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->d_work, c->s_comp, remote));
+  CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->d_work, c->s_comp, remote,
+                     timed && c->d_span ? c->d_span + c->kev_used : nullptr));
   if (timed) {
     CU(cudaEventRecord(c->kev[c->kev_used + 1], c->s_comp));
     c->kev_kind[c->kev_used / 2] = mode;
@@ -241,11 +245,19 @@ inline jitc_status run_segments(jitc_ctx* c, GroupState& g, int mode, const Laun
 
 // After the call's work has completed: harvest kernel timings into counters.
 inline void harvest(jitc_ctx* c) {
+  bool spans = c->d_span && c->kev_used &&
+               cudaMemcpyAsync(c->h_span.data(), c->d_span, c->kev_used * sizeof(unsigned long long),
+                               cudaMemcpyDeviceToHost, c->s_comp) == cudaSuccess &&
+               cudaStreamSynchronize(c->s_comp) == cudaSuccess;
   for (size_t i = 0; i + 1 < c->kev_used; i += 2) {
     float ms = 0;
     if (cudaEventElapsedTime(&ms, c->kev[i], c->kev[i + 1]) == cudaSuccess) {
       c->kc[c->kev_kind[i / 2]].ms += ms;
       c->kernel_ms_in_call += ms;
+    }
+    if (spans && c->h_span[i + 1]) {
+      const unsigned long long t0 = ~c->h_span[i], t1 = c->h_span[i + 1];
+      if (t1 > t0) c->kc[c->kev_kind[i / 2]].span_ms += (t1 - t0) * 1e-6;
     }
   }
   c->kev_used = 0;
@@ -263,8 +275,6 @@ inline void finish_stats(jitc_ctx* c, const CallTimer& t, jitc_stats* st, bool d
   }
 }
 
-// Segments whose image offset lies in [a, b) (segments never straddle a chunk
-// boundary and rounds are chunk-aligned, so this is exact).
 // A host<->device copy on `s`, issued in pieces of at most c->copy_piece bytes.
 inline cudaError_t copy_pieces(const jitc_ctx* c, void* dst, const void* src, uint64_t n, cudaMemcpyKind kind,
                                cudaStream_t s) {
@@ -277,6 +287,8 @@ inline cudaError_t copy_pieces(const jitc_ctx* c, void* dst, const void* src, ui
   return cudaSuccess;
 }
 
+// Segments whose image offset lies in [a, b) (segments never straddle a chunk
+// boundary and rounds are chunk-aligned, so this is exact).
 inline void seg_span(const GroupState& g, uint64_t a, uint64_t b, uint32_t* lo, uint32_t* hi) {
   auto cmp = [](const Seg& s, uint64_t v) { return s.img_off < v; };
   *lo = (uint32_t)(std::lower_bound(g.segs.begin(), g.segs.end(), a, cmp) - g.segs.begin());

@@ -72,8 +72,9 @@ struct LaunchRanges {
 // d_work: 2 x u32 zero-initialised device counters, private to the stream
 // (the kernel resets them when it finishes).
 // d_remote (kPull only): per-segment source address in a peer's memory.
-cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig,
-                            int grid, uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote = nullptr);
+cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig, int grid,
+                            uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote,
+                            unsigned long long* d_span = nullptr);
 cudaError_t launch_phase_write(uint64_t* dev_slot, uint64_t value, cudaStream_t s);
 int segment_grid(int device);
 cudaError_t device_check(int device, std::string* why);

@@ -118,11 +118,22 @@ __device__ __forceinline__ void flush(unsigned long long* dig, uint32_t chunk, u
 // zeroes it for the next launch on the stream.
 constexpr uint32_t kBatch = 8;
 
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// span (optional, timing diagnostics; zeroed before the launch): span[0] =
+// ~(first CTA start), span[1] = last CTA end, in %globaltimer nanoseconds
+// (the start is stored inverted so that both ends are an atomicMax).
 template <int MODE>
 __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ segs, LaunchRanges R,
                                                        unsigned long long* __restrict__ dig,
                                                        unsigned int* __restrict__ work,
-                                                       const uint64_t* __restrict__ remote) {
+                                                       const uint64_t* __restrict__ remote,
+                                                       unsigned long long* __restrict__ span) {
+  if (span && threadIdx.x == 0) atomicMax(span, ~gtimer());
   const uint32_t total = R.prefix[R.n];
   const uint32_t nbatch = (total + kBatch - 1) / kBatch;
   const int tid = threadIdx.x;
@@ -216,6 +227,10 @@ __global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ s
     }
   }
   if (cur_chunk != 0xFFFFFFFFu) flush(dig, cur_chunk, acc, lane);
+  if (span) {
+    __syncthreads();
+    if (tid == 0) atomicMax(span + 1, gtimer());
+  }
   // the last CTA out resets the counters for the next launch on this stream
   if (tid == 0) {
     __threadfence();
@@ -362,19 +377,19 @@ cudaError_t device_check(int device, std::string* why) {
 }
 
 cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig, int grid,
-                            uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote) {
+                            uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote, unsigned long long* d_span) {
   uint32_t total = r.prefix[r.n];
   if (total == 0) return cudaSuccess;
   uint32_t nbatch = (total + kBatch - 1) / kBatch;
   int g = (int)(nbatch < (uint32_t)grid ? nbatch : (uint32_t)grid);
   auto* dig = reinterpret_cast<unsigned long long*>(d_dig);
   switch (mode) {
-    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr); break;
-    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr); break;
-    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr); break;
+    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr, d_span); break;
+    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr, d_span); break;
+    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr, d_span); break;
     case kPull:
       if (!d_remote) return cudaErrorInvalidValue;
-      seg_kernel<kPull><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, d_remote);
+      seg_kernel<kPull><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, d_remote, d_span);
       break;
     default: return cudaErrorInvalidValue;
   }

@@ -62,7 +62,8 @@ class Stats(ctypes.Structure):
 
 
 class KernelCounter(ctypes.Structure):
-    _fields_ = [("launches", ctypes.c_uint64), ("bytes", ctypes.c_uint64), ("ms", ctypes.c_double)]
+    _fields_ = [("launches", ctypes.c_uint64), ("bytes", ctypes.c_uint64), ("ms", ctypes.c_double),
+                ("span_ms", ctypes.c_double)]
 
 
 _lib = None
@@ -490,7 +491,7 @@ class Context:
     def kernel_counters(self, kind: int) -> dict:
         kc = KernelCounter()
         _check(self._L.jitc_kernel_counters(self._h, kind, ctypes.byref(kc)), "jitc_kernel_counters")
-        return dict(launches=kc.launches, bytes=kc.bytes, ms=kc.ms)
+        return dict(launches=kc.launches, bytes=kc.bytes, ms=kc.ms, span_ms=kc.span_ms)
 
     def reset_counters(self):
         _check(self._L.jitc_reset_counters(self._h), "jitc_reset_counters")
