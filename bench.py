@@ -356,12 +356,30 @@ def run_jitc(args):
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms_step, ms_step_wall = tt.tolist()
 
+    # kernel counters of the timed region only (the extra variants below launch more)
+    kc_timed = {k: ctx.kernel_counters(k) for k in (J.K_DIGEST, J.K_PACK, J.K_UNPACK)}
+
+    # the paper's own protocol as an in-run comparison (
+    # PAPER.md:108, :136): every healthy rank saves its FULL state (k = 1 per
+    # rank, n * L over the host links) instead of a 1/k shard.  N > 1 only.
+    paper_protocol = None
+    if world > 1 and not args.no_paper_protocol:
+        dist.barrier()
+        t0 = time.perf_counter()
+        ctx.capture_local()
+        dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64)
+        dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+        paper_protocol = {"what": "every rank saves its full replica (own fingerprint, k=1 capture, commit); "
+                                  "host wall clock, max over ranks",
+                          "capture_s": round(dt.item(), 4), "host_link_bytes_total": world * L_total,
+                          "sharded_capture_s": round(statistics.median(per["capture"]) * 1e-3, 4),
+                          "sharded_host_link_bytes_total": L_total}
+
     # robustness variant: one more step while an emulated
     # hung collective (32 spinning CTAs on another stream) occupies the GPU,
     # as when a NCCL kernel waits forever on a dead peer
     under_hang = None
     if args.hang_ctas > 0:
-        kc_keep = {k: ctx.kernel_counters(k) for k in (J.K_DIGEST, J.K_PACK, J.K_UNPACK)}
         hs = torch.cuda.Stream()
         J.inject_hang(hs.cuda_stream, args.hang_ctas, slot=5)
         try:
@@ -378,7 +396,7 @@ def run_jitc(args):
 
     # roofline of the dominant kernel (largest total time in the timed region)
     kinds = {J.K_DIGEST: "K1_digest", J.K_PACK: "K2_pack_digest", J.K_UNPACK: "K3_unpack_verify"}
-    kc = kc_keep if under_hang is not None else {k: ctx.kernel_counters(k) for k in kinds}
+    kc = kc_timed
     dom = max(kc, key=lambda k: kc[k]["ms"])
     c = kc[dom]
     rw = 1 if dom == J.K_DIGEST else 2          # K1 reads L; K2/K3 read L and write L
@@ -436,6 +454,7 @@ def run_jitc(args):
                     "note": "host wall clock around the public Python API step (ctypes, manifest file I/O included)"},
             "gpu_launches": launches[0],
             "under_hang": under_hang,
+            "paper_protocol": paper_protocol,
             "clocks": clk.summary(),
         }
         if not args.no_cpu_baseline:
@@ -463,6 +482,8 @@ def main():
     ap.add_argument("--zero-copy", action="store_true")
     ap.add_argument("--image-dir", default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-paper-protocol", action="store_true",
+                    help="N > 1: skip the in-run comparison with the paper's every-rank-saves-everything protocol")
     ap.add_argument("--no-calibrate", action="store_true", help="skip the in-run host-link / HBM / NVLink calibration")
     ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],

@@ -123,6 +123,8 @@ void jitc_destroy(jitc_ctx* c) {
   if (c->s_comp) cudaStreamSynchronize(c->s_comp);
   if (c->s_copy) cudaStreamSynchronize(c->s_copy);
   if (c->comm) ncclCommDestroy(c->comm);
+  for (ncclComm_t r : c->retired_comms) ncclCommAbort(r);
+  c->retired_comms.clear();
   ipc_destroy(c);
   for (auto& kv : c->groups) free_group(kv.second);
   for (int i = 0; i < jitc_ctx::kSlots; ++i) {
@@ -361,8 +363,8 @@ jitc_status jitc_comm_init(jitc_ctx* c, const void* id128, int32_t nranks, int32
   if (!c || !id128 || nranks <= 0 || comm_rank < 0 || comm_rank >= nranks)
     return fail(JITC_EINVAL, "jitc_comm_init: bad argument");
   CU(cudaSetDevice(c->device));
-  if (c->comm) {
-    ncclCommDestroy(c->comm);
+  if (c->comm) {  // retired, not freed: see jitc_ctx::retired_comms
+    c->retired_comms.push_back(c->comm);
     c->comm = nullptr;
   }
   ncclUniqueId id;
@@ -400,9 +402,14 @@ jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_faile
     c->ipc->slot = slot;
     c->ipc->peer_staging = ps;
   } else {
+    // NCCL_SHRINK_ABORT aborts the parent's outstanding operations (a hung
+    // collective of this communicator exits); the parent itself is retired,
+    // not freed, until jitc_comm_destroy / jitc_destroy (see retired_comms).
     ncclComm_t nc = nullptr;
+    if (getenv("JITC_DEBUG_SHRINK")) fprintf(stderr, "jitc: ncclCommShrink ...\n");
     NC(ncclCommShrink(c->comm, excl.data(), (int)excl.size(), &nc, nullptr, NCCL_SHRINK_ABORT));
-    ncclCommAbort(c->comm);
+    if (getenv("JITC_DEBUG_SHRINK")) fprintf(stderr, "jitc: ncclCommShrink done\n");
+    c->retired_comms.push_back(c->comm);
     c->comm = nc;
   }
   std::vector<int32_t> job;
@@ -417,6 +424,8 @@ jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_faile
 jitc_status jitc_comm_destroy(jitc_ctx* c) {
   if (!c) return fail(JITC_EINVAL, "jitc_comm_destroy: null ctx");
   if (c->comm) ncclCommDestroy(c->comm);
+  for (ncclComm_t r : c->retired_comms) ncclCommAbort(r);
+  c->retired_comms.clear();
   c->comm = nullptr;
   ipc_destroy(c);
   c->comm_n = 0;

@@ -149,6 +149,10 @@ struct jitc_ctx {
   int grid = 0;
   // communicator
   ncclComm_t comm = nullptr;
+  // parents of jitc_comm_shrink, aborted but not yet freed: freeing device
+  // memory synchronises the device, and another communicator's collective
+  // (the framework's all-reduce) may still be hung on the dead rank
+  std::vector<ncclComm_t> retired_comms;
   int comm_n = 0, comm_rank = -1;
   std::vector<int32_t> comm_job;  // comm rank -> job rank
   std::unique_ptr<IpcComm> ipc;   // IPC transport (instead of `comm`)
@@ -361,8 +365,13 @@ inline int comm_rank_of(const jitc_ctx* c, int32_t job) {
   return -1;
 }
 
+// Writes `path` via a temp file + rename.  The temp name is unique per process
+// and call, so ranks that commit the same group at once (every rank's local
+// capture) never write into each other's temp file; the last
+// rename wins with a complete file.
 inline bool write_file_atomic(const std::string& path, const uint8_t* p, size_t n) {
-  std::string tmp = path + ".tmp";
+  static std::atomic<uint64_t> seq{0};
+  std::string tmp = path + ".tmp." + std::to_string((long)getpid()) + "." + std::to_string(seq++);
   FILE* f = fopen(tmp.c_str(), "wb");
   if (!f) return false;
   bool ok = fwrite(p, 1, n, f) == n;

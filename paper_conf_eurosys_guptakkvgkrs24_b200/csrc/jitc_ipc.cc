@@ -147,8 +147,8 @@ extern "C" jitc_status jitc_comm_init_ipc(jitc_ctx* c, const char* comm_dir, int
     return fail(JITC_EINVAL, "jitc_comm_init_ipc: bad argument");
   if (c->groups.size() > (size_t)kIpcMaxGroups) return fail(JITC_EINVAL, "jitc_comm_init_ipc: too many groups");
   CU(cudaSetDevice(c->device));
-  if (c->comm) {
-    ncclCommDestroy(c->comm);
+  if (c->comm) {  // retired, not freed: see jitc_ctx::retired_comms
+    c->retired_comms.push_back(c->comm);
     c->comm = nullptr;
   }
   ipc_destroy(c);
