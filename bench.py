@@ -394,6 +394,36 @@ def run_jitc(args):
                       "capture_GBps": round(cap_h["image_bytes"] / (cap_h["ms_host"] * 1e-3) / 1e9, 3),
                       "restore_GBps": round(res_h["image_bytes"] / (res_h["ms_host"] * 1e-3) / 1e9, 3)}
 
+    # communicator rebuild (SURVEY.md §8(d) d.6 T_comm; the paper's dominant
+    # recovery cost, Table 7): the survivors drop the last rank
+    # (jitc_comm_shrink), then all ranks build a fresh communicator including a
+    # "replacement" (jitc_comm_init / _ipc).  Host wall clock, max over ranks.
+    comm_rebuild = None
+    if world > 1 and not args.no_comm_rebuild:
+        victim = world - 1
+        dist.barrier()
+        t0 = time.perf_counter()
+        if rank != victim:
+            ctx.comm_shrink([victim])
+        t_shrink = time.perf_counter() - t0
+        dist.barrier()
+        if args.transport == "nccl":
+            uid = [J.get_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+        dist.barrier()
+        t0 = time.perf_counter()
+        if args.transport == "nccl":
+            ctx.comm_init(uid[0], world, rank)
+        else:
+            ctx.comm_init_ipc(f"{shm}-comm2", world, rank)
+        t_init = time.perf_counter() - t0
+        tt = torch.tensor([t_shrink, t_init], dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        comm_rebuild = {"transport": args.transport, "shrink_ms": round(tt[0].item() * 1e3, 2),
+                        "reinit_ms": round(tt[1].item() * 1e3, 2),
+                        "how": f"survivors shrink away rank {victim}, then all {world} ranks init a new "
+                               "communicator (warm-up included); host wall clock, max over ranks"}
+
     # roofline of the dominant kernel (largest total time in the timed region)
     kinds = {J.K_DIGEST: "K1_digest", J.K_PACK: "K2_pack_digest", J.K_UNPACK: "K3_unpack_verify"}
     kc = kc_timed
@@ -455,6 +485,7 @@ def run_jitc(args):
             "gpu_launches": launches[0],
             "under_hang": under_hang,
             "paper_protocol": paper_protocol,
+            "comm_rebuild": comm_rebuild,
             "clocks": clk.summary(),
         }
         if not args.no_cpu_baseline:
@@ -466,6 +497,7 @@ def run_jitc(args):
     if rank == 0 and not args.image_dir:
         shutil.rmtree(shm, ignore_errors=True)
         shutil.rmtree(f"{shm}-comm", ignore_errors=True)
+        shutil.rmtree(f"{shm}-comm2", ignore_errors=True)
 
 
 def main():
@@ -484,6 +516,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-paper-protocol", action="store_true",
                     help="N > 1: skip the in-run comparison with the paper's every-rank-saves-everything protocol")
+    ap.add_argument("--no-comm-rebuild", action="store_true", help="N > 1: skip timing shrink + re-init")
     ap.add_argument("--no-calibrate", action="store_true", help="skip the in-run host-link / HBM / NVLink calibration")
     ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],

@@ -359,6 +359,34 @@ jitc_status jitc_get_unique_id(void* id128) {
   return JITC_OK;
 }
 
+// One of each NCCL operation the library issues (all-gather of bytes and of
+// u64, the barrier's all-reduce, point-to-point send/recv), small and large,
+// right after the communicator is created.  The first collective of a process
+// does one-time work that waits behind a kernel already running on the device
+// -- measured: with no collective before a rank died, the survivors' first
+// all-gather after jitc_comm_shrink never started while an emulated hung
+// collective spun, and it ran at once when one collective had preceded the
+// failure (tools/debug_nccl_shrink.py) -- so it must happen here, in steady
+// state, never in the failure path (as with preload_kernels for our own).
+static jitc_status warm_comm(jitc_ctx* c) {
+  const uint64_t n = (uint64_t)c->comm_n, me = (uint64_t)c->comm_rank;
+  const uint64_t big = std::min<uint64_t>(1ull << 20, c->staging_bytes / (2 * n)) / 256 * 256;
+  for (uint64_t blk : {(uint64_t)256, big}) {
+    if (blk == 0 || n * blk > c->staging_bytes) continue;
+    NC(ncclAllGather(c->staging + me * blk, c->staging, blk, ncclUint8, c->comm, c->s_comp));
+    NC(ncclAllGather(c->staging + me * blk, c->staging, blk / 8, ncclUint64, c->comm, c->s_comp));
+    if (n > 1) {
+      NC(ncclGroupStart());
+      NC(ncclSend(c->staging, blk, ncclUint8, (int)((me + 1) % n), c->comm, c->s_comp));
+      NC(ncclRecv(c->staging + blk, blk, ncclUint8, (int)((me + n - 1) % n), c->comm, c->s_comp));
+      NC(ncclGroupEnd());
+    }
+  }
+  NC(ncclAllReduce(c->d_small, c->d_small + 1, 1, ncclUint64, ncclSum, c->comm, c->s_comp));
+  CU(cudaStreamSynchronize(c->s_comp));
+  return JITC_OK;
+}
+
 jitc_status jitc_comm_init(jitc_ctx* c, const void* id128, int32_t nranks, int32_t comm_rank, const int32_t* job_ranks) {
   if (!c || !id128 || nranks <= 0 || comm_rank < 0 || comm_rank >= nranks)
     return fail(JITC_EINVAL, "jitc_comm_init: bad argument");
@@ -376,7 +404,7 @@ jitc_status jitc_comm_init(jitc_ctx* c, const void* id128, int32_t nranks, int32
   for (int i = 0; i < nranks; ++i) c->comm_job[i] = job_ranks ? job_ranks[i] : i;
   if (c->comm_job[comm_rank] != c->cfg.rank)
     return fail(JITC_EINVAL, "jitc_comm_init: job_ranks[comm_rank] != cfg.rank");
-  return JITC_OK;
+  return warm_comm(c);
 }
 
 jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_failed) {
