@@ -148,3 +148,42 @@ def test_fanout_capture_tp2_dp2_lone_writer(transport):
         assert r.returncode == 0 and "replacement ok" in out, out
     finally:
         shutil.rmtree(shm, ignore_errors=True)
+
+
+def test_attach_image_and_fanout_argument_errors():
+    """jitc_attach_image is for declared (non-held) groups of a context with a
+    shared image_dir; jitc_capture_fanout needs a communicator."""
+    from paper_conf_eurosys_guptakkvgkrs24_b200 import build, jitc as J
+    from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
+    build.build()
+    shm = f"/dev/shm/jitc-fan-err-{os.getpid()}-{uuid.uuid4().hex[:8]}"
+    try:
+        g = W.scaled(W.c1(), 2000).groups[0]
+        st = GroupState(g, 5)
+        ctx = J.Context(device=0, rank=0, world=2, chunk_bytes=4096, image_dir=shm, staging_bytes=1 << 20,
+                        slot_bytes=1 << 18)
+        _, L = ctx.register(0, J.REQUIRED, [0, 1], st.table(), keepalive=st)
+        ctx.declare_group(1, J.OPTIONAL, [1])      # rank 1 is not healthy below: the group is dropped
+        with pytest.raises(J.JitcError):
+            ctx.attach_image(0, L)            # held: already has its image
+        with pytest.raises(J.JitcError):
+            ctx.attach_image(7, L)            # undeclared
+        with pytest.raises(J.JitcError):
+            ctx.attach_image(1, L + 1)        # not a multiple of 256
+        ctx.attach_image(1, L)
+        ctx.attach_image(1, L)                # idempotent
+        assert os.path.getsize(f"{shm}/g1.img") >= L
+        ctx.mark(0, 3, J.CLEAN)
+        blob = ctx.fingerprint()
+        s_, sel = J.select_consistent_replica(blob, [0])
+        assert s_ == J.OK, J.parse_selection(sel)
+        with pytest.raises(J.JitcError, match="communicator"):
+            ctx.capture_fanout(sel, [0])      # no communicator
+        ctx.close()
+        nodir = J.Context(device=0, rank=0, world=2, chunk_bytes=4096, staging_bytes=1 << 20, slot_bytes=1 << 18)
+        nodir.declare_group(1, J.REQUIRED, [1])
+        with pytest.raises(J.JitcError):
+            nodir.attach_image(1, L)          # private pinned images cannot be shared
+        nodir.close()
+    finally:
+        shutil.rmtree(shm, ignore_errors=True)

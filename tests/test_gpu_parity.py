@@ -281,14 +281,14 @@ def test_half_step_detected(J):
 def test_full_size_sampled(J, shm, cfg):
     """C2 (GPT-2 1.5B, 24.9 GB) and C3 (Llama-3-8B, 128.5 GB, the BASELINE
     target shape) in the launch configuration bench.py times (1 MiB chunks,
-    2 GiB rounds, 8 GiB staging): K1 digests of sampled chunks equal the
+    4 GiB rounds, 8 GiB staging): K1 digests of sampled chunks equal the
     oracle's (computed chunk by chunk), the packed image bytes of those chunks
     equal the oracle's, and capture -> restore -> verify round-trips."""
     w = W.CONFIGS[cfg]()
     C = 1 << 20
     states = {g.group: _state(g, w.seed) for g in w.groups}
     ctx = J.Context(device=0, chunk_bytes=C, image_dir=shm, flags=J.F_TIME_KERNELS, staging_bytes=8 << 30,
-                    slot_bytes=2 << 30)
+                    slot_bytes=4 << 30)
     for g in w.groups:
         ctx.register(g.group, g.policy, [0], states[g.group].table(), keepalive=states[g.group])
         ctx.mark(g.group, 100, J.CLEAN)
