@@ -394,6 +394,34 @@ def run_jitc(args):
                       "capture_GBps": round(cap_h["image_bytes"] / (cap_h["ms_host"] * 1e-3) / 1e9, 3),
                       "restore_GBps": round(res_h["image_bytes"] / (res_h["ms_host"] * 1e-3) / 1e9, 3)}
 
+    # NEXT-1: the native watchdog detects
+    # an emulated hung collective and captures on its own thread.  N = 1 only:
+    # waited = event age when the watchdog fired (>= the timeout), action =
+    # fingerprint -> select -> capture -> commit run by the watchdog thread.
+    on_hang = None
+    if world == 1 and args.hang_ctas > 0 and not args.no_watchdog:
+        hs = torch.cuda.Stream()
+        J.inject_hang(hs.cuda_stream, args.hang_ctas, slot=6)
+        ev = torch.cuda.Event()
+        ev.record(hs)
+        try:
+            ctx.watch_event(ev.cuda_event, tag=7)
+            ctx.watchdog_start(timeout_ms=args.watchdog_ms, action=J.ON_HANG_LOCAL_CAPTURE)
+            r = ctx.watchdog_wait(120000)
+        finally:
+            J.inject_release(6)
+        hs.synchronize()
+        ctx.watchdog_stop()
+        st_w = r["stats"]
+        on_hang = {"timeout_ms": args.watchdog_ms, "fired": r["fired"], "waited_ms": round(r["waited_ms"], 2),
+                   "detect_overshoot_ms": round(r["waited_ms"] - args.watchdog_ms, 2),
+                   "action_ms": round(r["action_ms"], 1),
+                   "capture_GBps": round(st_w["image_bytes"] / (r["action_ms"] * 1e-3) / 1e9, 2)
+                   if r["action_ms"] else None,
+                   "hung_ctas": args.hang_ctas,
+                   "how": "jitc_watchdog_start(ON_HANG_LOCAL_CAPTURE) on an event after spinning CTAs; the "
+                          "action (fingerprint, own select, capture, commit) runs on the watchdog thread"}
+
     # communicator rebuild (SURVEY.md §8(d) d.6 T_comm; the paper's dominant
     # recovery cost, Table 7): the survivors drop the last rank
     # (jitc_comm_shrink), then all ranks build a fresh communicator including a
@@ -486,6 +514,7 @@ def run_jitc(args):
             "under_hang": under_hang,
             "paper_protocol": paper_protocol,
             "comm_rebuild": comm_rebuild,
+            "watchdog_on_hang": on_hang,
             "clocks": clk.summary(),
         }
         if not args.no_cpu_baseline:
@@ -516,6 +545,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-paper-protocol", action="store_true",
                     help="N > 1: skip the in-run comparison with the paper's every-rank-saves-everything protocol")
+    ap.add_argument("--no-watchdog", action="store_true", help="N = 1: skip the watchdog on-hang capture variant")
+    ap.add_argument("--watchdog-ms", type=int, default=200, help="watchdog hang timeout for that variant")
     ap.add_argument("--no-comm-rebuild", action="store_true", help="N > 1: skip timing shrink + re-init")
     ap.add_argument("--no-calibrate", action="store_true", help="skip the in-run host-link / HBM / NVLink calibration")
     ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
