@@ -1,6 +1,6 @@
 """Host-code sanitizers: the pure C-ABI functions -- replica
-selection, blob / selection parsing, layout, shard rule, restore plans, the
-analytic model -- run under AddressSanitizer + UndefinedBehaviorSanitizer in
+selection, blob / selection parsing, layout, shard rule, restore and capture
+(fan-out) plans, the analytic model -- run under AddressSanitizer + UndefinedBehaviorSanitizer in
 a child process that loads libjitc_asan.so (same sources, host code
 instrumented), including malformed and truncated inputs."""
 import os
@@ -44,6 +44,12 @@ for trial in range(400):
             for mode in (0, 1):
                 for me in range(world):
                     J.restore_plan(sel, e.group, mode, list(range(world)), me, 8 * 4096 * 4, 2 * 4096)
+            movers = sorted(rnd.sample(healthy, rnd.randint(1, len(healthy))))
+            for me in range(len(healthy)):
+                try:
+                    J.capture_plan(sel, e.group, movers, healthy, me, rnd.choice([4096, 8 * 4096 * 4]), 2 * 4096)
+                except J.JitcError:
+                    pass         # staging below 2 * k * C, or a writer outside the communicator
     # malformed inputs: truncations and bit flips must be rejected, never crash
     for cut in (1, 7, 31, 33, 64, len(buf) // 2, len(buf) - 1):
         if 0 < cut < len(buf):
