@@ -175,3 +175,17 @@ def test_select_random_record_sets_match_oracle(J):
 def test_select_rejects_garbage(J):
     st = J.lib().jitc_select_consistent_replica(b"\0" * 40, 40, None, 0, None, 0, None)
     assert st == J.EINVAL
+
+
+def test_select_exhaustive_small_worlds_match_oracle(J):
+    """The C ABI's selection equals the oracle's on every small-world pure-DP
+    scenario of the brute-force pin (tests/test_oracle_select.py)."""
+    import tests.test_oracle_select as T
+    n = 0
+    for states in T.small_world_scenarios():
+        buf, healthy = T.scenario_buffer(states)
+        if not buf:
+            continue
+        _compare(J, buf, healthy)
+        n += 1
+    assert n > 10000

@@ -64,23 +64,29 @@ def test_uncommitted_refused():
 
 def test_half_step_detected():
     """A half-applied optimizer step (U_v on tensors [0, split)) changes the
-    digests of exactly the chunks those tensors touch."""
+    digests of exactly the chunks those tensors touch -- at
+    every split point, built incrementally: split s+1
+    is split s plus the update of tensor s."""
     w = _c1_small()
     g = w.groups[0]
     lay = O.layout_of_group(g, 4096)
     ts = O.gen_group(g, w.seed)
     d0 = O.jf64(O.pack(ts, lay), lay.C, 0, lay.n_c)
     L = O.lib()
-    for split in range(1, len(ts), 17):
-        t2 = [t.copy() for t in ts]
-        for i in range(split):
-            if g.tensors[i].dtype == "f32":
-                x = t2[i].view(np.uint32)
-                L.orc_update_fp32(O._ptr(x), 0, len(x), g.tensors[i].gen_id, 4)
-        d1 = O.jf64(O.pack(t2, lay), lay.C, 0, lay.n_c)
-        touched = set()
-        for i in range(split):
+    t2 = [t.copy() for t in ts]
+    touched = set()
+    n_split = 0
+    for split in range(1, len(ts) + 1):
+        i = split - 1
+        if g.tensors[i].dtype == "f32":
+            x = t2[i].view(np.uint32)
+            L.orc_update_fp32(O._ptr(x), 0, len(x), g.tensors[i].gen_id, 4)
             touched |= set(range(lay.offsets[i] // lay.C, (lay.offsets[i] + lay.nbytes[i] - 1) // lay.C + 1))
+        if split == len(ts):
+            break                       # the whole step applied: not a half step
+        d1 = O.jf64(O.pack(t2, lay), lay.C, 0, lay.n_c)
         changed = set(np.nonzero(d0 != d1)[0].tolist())
-        assert changed == touched
-        assert O.root(lay.layout_hash, d0) != O.root(lay.layout_hash, d1)
+        assert changed == touched, split
+        assert (O.root(lay.layout_hash, d0) != O.root(lay.layout_hash, d1)) == bool(touched), split
+        n_split += 1
+    assert n_split == len(ts) - 1

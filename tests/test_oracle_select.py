@@ -217,3 +217,100 @@ def test_record_blob_roundtrip():
     for a, b in zip(rs, r2):
         assert (a.group, a.version, a.root, a.L) == (b.group, b.version, b.root, b.L)
         assert np.array_equal(a.d, b.d)
+
+
+# ----------------------------------------------------------------------------
+# Brute force over small worlds: every pure-DP
+# scenario with n <= 4 ranks (and every n = 5 scenario with both i and i+1
+# present), each rank dead or alive x version {i, i+1} x phase {CLEAN, DIRTY}
+# x corrupted {no, yes}, at most 2 corrupted ranks.  The expectation is not
+# the oracle's step-by-step procedure: it is the closed-form statement of the
+# rule for one group, written from the paper's cases --
+#   * a state is restorable iff it is CLEAN (PAPER.md:184-188 hooks) and held
+#     by a strict plurality of identical CLEAN replicas of that minibatch
+#     ("discard corrupted"; reading R8: ties are conflicts);
+#   * among restorable minibatches the newest wins;
+#   * nothing restorable: a conflict if any CLEAN replica exists (then every
+#     version present is tied), else no consistent state (all DIRTY);
+#   * nobody alive: no replica.
+# A dead rank contributes nothing; a corrupted rank's bytes are its own.
+# ----------------------------------------------------------------------------
+_DEAD = None
+
+
+def _rank_states():
+    yield _DEAD
+    for v in (I, I + 1):
+        for ph in (O.CLEAN, O.DIRTY):
+            for bad in (False, True):
+                yield (v, ph, bad)
+
+
+def _expected_single_group(states):
+    alive = {r: s for r, s in enumerate(states) if s is not _DEAD}
+    if not alive:
+        return O.ENOREPLICA, None, None, None
+    content = {r: (v, r if bad else -1) for r, (v, ph, bad) in alive.items()}
+    clean = [r for r, (v, ph, bad) in alive.items() if ph == O.CLEAN]
+    best = {}
+    for v in {alive[r][0] for r in clean}:
+        holders = {}
+        for r in clean:
+            if alive[r][0] == v:
+                holders.setdefault(content[r], []).append(r)
+        counts = sorted((len(h) for h in holders.values()), reverse=True)
+        if len(counts) == 1 or counts[0] > counts[1]:
+            best[v] = sorted(max(holders.values(), key=len))
+    if not best:
+        return (O.ECONFLICT if clean else O.ENOCONSISTENT), None, None, None
+    vs = max(best)
+    writers = best[vs]
+    reasons = {}
+    for r, (v, ph, bad) in alive.items():
+        if r in writers:
+            continue
+        reasons[r] = O.R_DIRTY if ph == O.DIRTY else (O.R_STALE_VERSION if v != vs else O.R_MINORITY)
+    return O.OK, vs, writers, reasons
+
+
+def small_world_scenarios(max_n=4, n5=True):
+    import itertools
+    for n in range(1, max_n + 1):
+        for states in itertools.product(list(_rank_states()), repeat=n):
+            if sum(1 for s in states if s is not _DEAD and s[2]) <= 2:
+                yield states
+    if n5:
+        for states in itertools.product(list(_rank_states()), repeat=5):
+            alive = [s for s in states if s is not _DEAD]
+            if sum(1 for s in alive if s[2]) <= 2 and {s[0] for s in alive} == {I, I + 1} \
+                    and sum(1 for s in alive if s[1] == O.DIRTY) <= 1:
+                yield states
+
+
+def scenario_buffer(states):
+    n = len(states)
+    topo = dp_topo(n)
+    rb = {}
+    for r, s in enumerate(states):
+        if s is _DEAD:
+            continue
+        v, ph, bad = s
+        rb[r] = [rec(r, 0, v, phase=ph, content=(5000 + 10 * r + v) if bad else v)]
+    return blobs(topo, rb) if rb else b"", sorted(rb)
+
+
+def test_select_exhaustive_small_worlds():
+    count = 0
+    for states in small_world_scenarios():
+        buf, healthy = scenario_buffer(states)
+        st, vs, writers, reasons = _expected_single_group(states)
+        sel = O.select(buf, healthy) if buf else O.select(b"", [])
+        assert sel.status == st, states
+        count += 1
+        if st != O.OK:
+            continue
+        g = gsel(sel, 0)
+        assert sel.v_star == vs and g.writers == writers, states
+        assert g.status == (O.G_UNVERIFIED_SINGLE if len(writers) == 1 else O.G_OK), states
+        assert dict(g.excluded) == reasons, states
+    assert count > 10000          # 14,430 scenarios
