@@ -81,7 +81,7 @@ int main(int argc, char** argv) {
       r.base[0] = (uint64_t)stage;
       r.base_off[0] = (uint64_t)base * seg_bytes;
       if (each) CK(cudaEventRecord(ev[2 + 2 * j], s));
-      CK(launch_segments(mode, d_segs, r, dig, grid, work, s));
+      CK(launch_segments(mode, d_segs, r, dig, grid, work, s, nullptr, nullptr));
       if (each) CK(cudaEventRecord(ev[3 + 2 * j], s));
     }
     CK(cudaEventRecord(ev[1], s));
