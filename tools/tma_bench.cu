@@ -144,6 +144,73 @@ __global__ void __launch_bounds__(kT) tma_pack(const uint8_t* __restrict__ src, 
   if (tid == 0) bulk_wait_all();
 }
 
+// tma_pack_warp: the same pipeline per WARP instead of per CTA -- every warp
+// owns a private S-stage ring of W-byte tiles in shared memory, lane 0 issues
+// its bulk loads/stores, and the only synchronisation is __syncwarp and the
+// warp's own mbarriers (no CTA-wide barrier per tile).
+template <uint32_t W, int S>
+__global__ void __launch_bounds__(kT) tma_pack_warp(const uint8_t* __restrict__ src, uint8_t* __restrict__ dst,
+                                                    uint64_t ntiles, uint64_t img0, uint64_t C,
+                                                    unsigned long long* __restrict__ dig) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) uint64_t full[kT / 32][S];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint8_t* ring = smem + (size_t)wid * S * W;
+  if (lane == 0) {
+    for (int s = 0; s < S; ++s) mbar_init(&full[wid][s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  const uint64_t nw = (uint64_t)gridDim.x * (kT / 32);
+  const uint64_t gw = (uint64_t)blockIdx.x * (kT / 32) + wid;
+  const uint64_t n = gw < ntiles ? (ntiles - gw + nw - 1) / nw : 0;
+  auto tile_of = [&](uint64_t i) { return gw + i * nw; };
+  if (lane == 0)
+    for (uint64_t i = 0; i < (uint64_t)(S - 1) && i < n; ++i) {
+      mbar_expect_tx(&full[wid][i], W);
+      bulk_load(ring + i * W, src + tile_of(i) * W, W, &full[wid][i]);
+    }
+  for (uint64_t i = 0; i < n; ++i) {
+    const int s = (int)(i % S);
+    mbar_wait(&full[wid][s], (uint32_t)((i / S) & 1));
+    const uint64_t t = tile_of(i);
+    const uint64_t off = img0 + t * W;
+    const uint4* in = reinterpret_cast<const uint4*>(ring + s * W);
+    uint64_t acc = 0;
+#pragma unroll
+    for (int u = 0; u < (int)(W / 16 / 32); ++u) {
+      const uint32_t v = lane + u * 32;
+      const uint4 x = in[v];
+      const uint64_t key = ((off >> 3) + 2ull * v + 1ull) * kPhi;
+      acc += mix(((uint64_t)x.x | ((uint64_t)x.y << 32)) ^ key);
+      acc += mix(((uint64_t)x.z | ((uint64_t)x.w << 32)) ^ (key + kPhi));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) {
+      atomicAdd(dig + off / C, (unsigned long long)acc);
+      bulk_store(dst + t * W, ring + s * W, W);
+      bulk_commit();
+      const uint64_t nx = i + S - 1;
+      if (nx < n) {
+        bulk_wait_read<1>();
+        const int s2 = (int)(nx % S);
+        mbar_expect_tx(&full[wid][s2], W);
+        bulk_load(ring + s2 * W, src + tile_of(nx) * W, W, &full[wid][s2]);
+      }
+    }
+    __syncwarp();
+  }
+  if (lane == 0) bulk_wait_all();
+}
+
+struct Variant {
+  const char* name;
+  const void* fn;
+  size_t smem;
+  uint32_t tile;
+};
+
 int main(int argc, char** argv) {
   const uint64_t launch_bytes = (uint64_t)(argc > 1 ? atoll(argv[1]) : 4096) << 20;
   const uint64_t arena_bytes = (uint64_t)(argc > 2 ? atoll(argv[2]) : 16384) << 20;
@@ -192,17 +259,29 @@ int main(int argc, char** argv) {
   CK(cudaMalloc(&work, 64));
   CK(cudaMemset(work, 0, 64));
   const int seg_grid = segment_grid(0);
-  const size_t smem = kStages * kTile;
-  CK(cudaFuncSetAttribute(tma_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int per_sm = 0, sms = 0;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tma_pack, kT, smem));
+  int sms = 0;
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
-  const int tma_grid = sms * per_sm;
   const uint32_t nl = (uint32_t)(arena_bytes / launch_bytes);
   const uint32_t per = (uint32_t)(launch_bytes / seg_bytes);
-  printf("launch %llu MiB, arena %llu MiB, %u launches; seg_kernel grid %d; tma_pack grid %d (%d/SM, %zu B smem)\n",
-         (unsigned long long)(launch_bytes >> 20), (unsigned long long)(arena_bytes >> 20), nl, seg_grid, tma_grid,
-         per_sm, smem);
+  printf("launch %llu MiB, arena %llu MiB, %u launches; seg_kernel grid %d\n",
+         (unsigned long long)(launch_bytes >> 20), (unsigned long long)(arena_bytes >> 20), nl, seg_grid);
+
+  std::vector<Variant> vs = {
+      {"tma_pack CTA ring 4 x 16 KiB", (const void*)tma_pack, kStages * kTile, kTile},
+      {"tma_pack_warp 4 x 4 KiB per warp", (const void*)tma_pack_warp<4096, 4>, 8 * 4 * 4096, 4096},
+      {"tma_pack_warp 6 x 4 KiB per warp", (const void*)tma_pack_warp<4096, 6>, 8 * 6 * 4096, 4096},
+      {"tma_pack_warp 3 x 8 KiB per warp", (const void*)tma_pack_warp<8192, 3>, 8 * 3 * 8192, 8192},
+      {"tma_pack_warp 8 x 2 KiB per warp", (const void*)tma_pack_warp<2048, 8>, 8 * 8 * 2048, 2048},
+      {"tma_pack_warp 12 x 2 KiB per warp", (const void*)tma_pack_warp<2048, 12>, 8 * 12 * 2048, 2048},
+  };
+  std::vector<int> grids;
+  for (auto& v : vs) {
+    CK(cudaFuncSetAttribute(v.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem));
+    int per_sm = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, v.fn, kT, v.smem));
+    grids.push_back(sms * per_sm);
+    printf("  %-36s smem %6zu B  %d CTA/SM  grid %d\n", v.name, v.smem, per_sm, sms * per_sm);
+  }
 
   auto launch_seg = [&](uint32_t j) {
     LaunchRanges r{};
@@ -214,43 +293,51 @@ int main(int argc, char** argv) {
     r.base_off[0] = (uint64_t)j * launch_bytes;
     CK(launch_segments(kPack, d_segs, r, dig_a, seg_grid, work, s, nullptr, nullptr));
   };
-  auto launch_tma = [&](uint32_t j) {
-    tma_pack<<<tma_grid, kT, smem, s>>>(src + (uint64_t)j * launch_bytes, stage_b, launch_bytes / kTile,
-                                        (uint64_t)j * launch_bytes, C, (unsigned long long*)dig_b);
-    CK(cudaGetLastError());
+  auto launch_var = [&](int k, uint32_t j) {
+    const uint8_t* a0 = src + (uint64_t)j * launch_bytes;
+    uint8_t* a1 = stage_b;
+    uint64_t a2 = launch_bytes / vs[k].tile, a3 = (uint64_t)j * launch_bytes, a4 = C;
+    unsigned long long* a5 = (unsigned long long*)dig_b;
+    void* args[] = {&a0, &a1, &a2, &a3, &a4, &a5};
+    CK(cudaLaunchKernel(vs[k].fn, dim3(grids[k]), dim3(kT), args, vs[k].smem, s));
   };
 
-  // correctness: the last launch's staging bytes and all digests
+  // correctness of every variant: all digests and the last launch's staging bytes
+  bool all_ok = true;
   CK(cudaMemset(dig_a, 0, nch * 8));
-  CK(cudaMemset(dig_b, 0, nch * 8));
-  for (uint32_t j = 0; j < nl; ++j) {
-    launch_seg(j);
-    launch_tma(j);
-  }
+  for (uint32_t j = 0; j < nl; ++j) launch_seg(j);
   CK(cudaStreamSynchronize(s));
   std::vector<uint64_t> da(nch), db(nch);
   CK(cudaMemcpy(da.data(), dig_a, nch * 8, cudaMemcpyDeviceToHost));
-  CK(cudaMemcpy(db.data(), dig_b, nch * 8, cudaMemcpyDeviceToHost));
-  const bool dig_ok = da == db;
   std::vector<uint8_t> sa(64 << 20), sb(64 << 20);
-  bool img_ok = true;
-  for (uint64_t o = 0; o < launch_bytes; o += sa.size()) {
-    CK(cudaMemcpy(sa.data(), stage_a + o, sa.size(), cudaMemcpyDeviceToHost));
-    CK(cudaMemcpy(sb.data(), stage_b + o, sb.size(), cudaMemcpyDeviceToHost));
-    img_ok &= memcmp(sa.data(), sb.data(), sa.size()) == 0;
+  for (size_t k = 0; k < vs.size(); ++k) {
+    CK(cudaMemset(dig_b, 0, nch * 8));
+    CK(cudaMemset(stage_b, 0, launch_bytes));
+    for (uint32_t j = 0; j < nl; ++j) launch_var((int)k, j);
+    CK(cudaStreamSynchronize(s));
+    CK(cudaMemcpy(db.data(), dig_b, nch * 8, cudaMemcpyDeviceToHost));
+    const bool dig_ok = da == db;
+    bool img_ok = true;
+    for (uint64_t o = 0; o < launch_bytes; o += sa.size()) {
+      CK(cudaMemcpy(sa.data(), stage_a + o, sa.size(), cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(sb.data(), stage_b + o, sb.size(), cudaMemcpyDeviceToHost));
+      img_ok &= memcmp(sa.data(), sb.data(), sa.size()) == 0;
+    }
+    printf("%-36s == seg_kernel<kPack>: digests %s, staging bytes %s\n", vs[k].name, dig_ok ? "equal" : "DIFFER",
+           img_ok ? "equal" : "DIFFER");
+    all_ok &= dig_ok && img_ok;
   }
-  printf("tma_pack == seg_kernel<kPack>: digests %s, staging bytes %s\n", dig_ok ? "equal" : "DIFFER",
-         img_ok ? "equal" : "DIFFER");
 
   std::vector<cudaEvent_t> ev(2 * nl);
   for (auto& e : ev) CK(cudaEventCreate(&e));
-  auto timed = [&](const char* name, bool tma, bool d2h) {
+  const uint64_t d2h_bytes = 4ull << 30;   // from the (>= 4 GiB) source arena
+  auto timed = [&](const char* name, int k, bool d2h) {
     double best = 1e30;
     for (int rep = 0; rep < 3; ++rep) {
-      if (d2h) CK(cudaMemcpyAsync(host, stage_a, 4ull << 30, cudaMemcpyDeviceToHost, s2));
+      if (d2h) CK(cudaMemcpyAsync(host, src, d2h_bytes, cudaMemcpyDeviceToHost, s2));
       for (uint32_t j = 0; j < nl; ++j) {
         CK(cudaEventRecord(ev[2 * j], s));
-        tma ? launch_tma(j) : launch_seg(j);
+        k < 0 ? launch_seg(j) : launch_var(k, j);
         CK(cudaEventRecord(ev[2 * j + 1], s));
       }
       CK(cudaStreamSynchronize(s));
@@ -263,12 +350,12 @@ int main(int argc, char** argv) {
       }
       best = sum / nl < best ? sum / nl : best;
     }
-    printf("%-40s %8.1f us/launch  %7.0f GB/s (read+write)\n", name, best * 1e3,
+    printf("%-36s %s %8.1f us/launch  %7.0f GB/s (read+write)\n", name, d2h ? "+D2H" : "    ", best * 1e3,
            2.0 * launch_bytes / (best * 1e-3) / 1e9);
   };
-  timed("seg_kernel<kPack> (LDG.128/STG.128)", false, false);
-  timed("tma_pack (cp.async.bulk 16 KiB tiles)", true, false);
-  timed("seg_kernel<kPack> + concurrent D2H", false, true);
-  timed("tma_pack + concurrent D2H", true, true);
-  return dig_ok && img_ok ? 0 : 2;
+  for (int d2h = 0; d2h < 2; ++d2h) {
+    timed("seg_kernel<kPack> (LDG.128/STG.128)", -1, d2h);
+    for (size_t k = 0; k < vs.size(); ++k) timed(vs[k].name, (int)k, d2h);
+  }
+  return all_ok ? 0 : 2;
 }
