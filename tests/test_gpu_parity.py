@@ -348,6 +348,58 @@ def test_edge_empty_tensors_empty_group_max_chunk(J, shm):
         shutil.rmtree(d, ignore_errors=True)
 
 
+@pytest.mark.slow
+def test_edge_tensors_over_4gib(J, shm):
+    """Maximum sizes: two tensors larger than 4 GiB (a u8 one of 4 GiB + 5 B
+    at a 2-byte-misaligned address, an fp32 one of 4 GiB + 12 B -- the size
+    class of an unsharded 70B-model embedding in fp32), so every 32-bit
+    element, byte and segment count would wrap.  1 MiB chunks, 1 GiB rounds.
+    Sampled chunks around each 4 GiB boundary, the tails and the first chunk
+    equal the oracle's image bytes and digests; the restore is bit-exact on
+    the same samples and verify passes over the whole group."""
+    big = 1 << 32
+    g = W.GroupSpec(3, J.REQUIRED, [0], [
+        W.TensorSpec("head", "f32", 1000, "master", 0),
+        W.TensorSpec("emb.u8", "u8", big + 5, "bytes", 1),
+        W.TensorSpec("emb.f32", "f32", (big + 12) // 4, "master", 2),
+        W.TensorSpec("tail", "bf16", 777, "master", 3),
+    ])
+    C = 1 << 20
+    st = _state(g, 9, misalign=2)
+    assert st.ptrs[1] % 16 == 2
+    ctx = _ctx(J, C, image_dir=shm, staging=2 << 30, slot=1 << 30)
+    lh, L = ctx.register(3, J.REQUIRED, [0], st.table(), keepalive=st)
+    lay = O.layout_of_group(g, C)
+    assert (lh, L) == (lay.layout_hash, lay.L) and L > 2 * big
+    blob, sel, cap = _pipeline(J, ctx)
+    rec = _records(blob)[3]
+    marks = [0, lay.L - 1]
+    for i in (1, 2):
+        marks += [lay.offsets[i], lay.offsets[i] + big - 1, lay.offsets[i] + big, lay.offsets[i] + g.tensors[i].nbytes - 1]
+    chunks = sorted({m // C for m in marks} | {m // C + 1 for m in marks if m // C + 1 < lay.n_c})
+    img = np.memmap(f"{shm}/g3.img", dtype=np.uint8, mode="r")
+    want = {}
+    for c in chunks:
+        a, b = c * C, min((c + 1) * C, lay.L)
+        want[c] = O.image_range(g, 9, lay, a, b)
+        assert np.array_equal(np.asarray(img[a:b]), want[c]), c
+        assert int(rec.d[c]) == int(O.jf64(want[c], C, a, lay.n_c)[c]), c
+    st.scramble()
+    ctx.restore(3, J.HOST)
+    ctx.verify(3, blob)
+    torch.cuda.synchronize()
+    for c in chunks:
+        a, b = c * C, min((c + 1) * C, lay.L)
+        for i, t in enumerate(g.tensors):
+            lo, hi = max(a, lay.offsets[i]), min(b, lay.offsets[i] + t.nbytes)
+            if lo < hi:
+                got = st.tensor_bytes(i)[lo - lay.offsets[i]:hi - lay.offsets[i]].cpu().numpy()
+                assert np.array_equal(got, want[c][lo - a:hi - a]), (c, t.name)
+    ctx.close()
+    del st
+    torch.cuda.empty_cache()
+
+
 def test_layout_mismatch_between_replicas(J):
     """S10 with real fingerprints: one replica registered one tensor with a
     different size -> ELAYOUT for the whole selection."""
