@@ -203,37 +203,91 @@ def image_range(g, seed: int, lay: Layout, a: int, b: int) -> np.ndarray:
 # ----------------------------------------------------------------------------
 # O2 pack / O8 unpack
 # ----------------------------------------------------------------------------
-def pack(tensors: Sequence[np.ndarray], lay: Layout) -> np.ndarray:
+def _parts(n: int, threads: int) -> List[Tuple[int, int]]:
+    """[0, n) cut into `threads` contiguous, nearly equal parts (O5's rule)."""
+    t = max(1, min(threads, n)) if n else 1
+    return [(s * n // t, (s + 1) * n // t) for s in range(t)]
+
+
+def _run_parts(fn, parts):
+    """Runs fn(a, b) for every part; with more than one part, on threads
+    (ctypes releases the GIL inside the C calls).  The parts touch disjoint
+    bytes, so the result is the single-threaded one."""
+    if len(parts) == 1:
+        fn(*parts[0])
+        return
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(len(parts)) as ex:
+        list(ex.map(lambda ab: fn(*ab), parts))
+
+
+def pack(tensors: Sequence[np.ndarray], lay: Layout, threads: int = 1) -> np.ndarray:
+    """O2.  threads > 1 (oracle timing): tensors are cut
+    into contiguous runs and each run is packed into its own image span
+    [off[first], off[last+1]) -- the spans partition [0, L)."""
     img = np.empty(lay.L, dtype=np.uint8)
     ts = [np.ascontiguousarray(t) for t in tensors]
-    src = (ctypes.c_void_p * len(ts))(*[_ptr(t) for t in ts])
+    src = (ctypes.c_void_p * max(1, len(ts)))(*[_ptr(t) for t in ts])
     nb = np.array(lay.nbytes, dtype=np.uint64)
     off = np.array(lay.offsets, dtype=np.uint64)
-    lib().orc_pack(src, _ptr(nb), _ptr(off), len(ts), _ptr(img), lay.L)
+    ends = list(lay.offsets[1:]) + [lay.L]
+
+    def run(a, b):
+        if a == b:
+            return
+        base = lay.offsets[a]
+        rel = off[a:b] - np.uint64(base)
+        sub = (ctypes.c_void_p * (b - a))(*[src[i] for i in range(a, b)])
+        lib().orc_pack(sub, _ptr(nb[a:b]), _ptr(rel), b - a, _ptr(img) + base, ends[b - 1] - base)
+
+    if not ts:
+        img[:] = 0
+    else:
+        _run_parts(run, _parts(len(ts), threads))
     return img
 
 
-def unpack(img: np.ndarray, lay: Layout) -> List[np.ndarray]:
+def unpack(img: np.ndarray, lay: Layout, threads: int = 1) -> List[np.ndarray]:
+    """O8 unpack; threads > 1 splits the tensor list (disjoint destinations)."""
     outs = [np.empty(nb, dtype=np.uint8) for nb in lay.nbytes]
-    dst = (ctypes.c_void_p * len(outs))(*[_ptr(t) for t in outs])
+    dst = (ctypes.c_void_p * max(1, len(outs)))(*[_ptr(t) for t in outs])
     nb = np.array(lay.nbytes, dtype=np.uint64)
     off = np.array(lay.offsets, dtype=np.uint64)
-    lib().orc_unpack(_ptr(img), dst, _ptr(nb), _ptr(off), len(outs))
+
+    def run(a, b):
+        if a == b:
+            return
+        sub = (ctypes.c_void_p * (b - a))(*[dst[i] for i in range(a, b)])
+        lib().orc_unpack(_ptr(img), sub, _ptr(nb[a:b]), _ptr(off[a:b]), b - a)
+
+    if outs:
+        _run_parts(run, _parts(len(outs), threads))
     return outs
 
 
 # ----------------------------------------------------------------------------
 # O3 JF64
 # ----------------------------------------------------------------------------
-def jf64(img: np.ndarray, C: int, byte0: int = 0, n_c: Optional[int] = None) -> np.ndarray:
+def jf64(img: np.ndarray, C: int, byte0: int = 0, n_c: Optional[int] = None, threads: int = 1) -> np.ndarray:
     """Chunk digests of an image fragment starting at image byte byte0 (a
-    multiple of 8); returns d indexed by global chunk id (length n_c)."""
+    multiple of 8); returns d indexed by global chunk id (length n_c).
+    threads > 1 (oracle timing): the fragment is cut at
+    chunk boundaries, so every thread owns whole digests d[c]."""
     assert img.dtype == np.uint8 and len(img) % 8 == 0 and byte0 % 8 == 0
     if n_c is None:
         n_c = (byte0 + len(img) + C - 1) // C
     d = np.zeros(n_c, dtype=np.uint64)
     img = np.ascontiguousarray(img)
-    lib().orc_jf64_accumulate(_ptr(img), byte0 // 8, len(img) // 8, C // 8, _ptr(d))
+    g0, nw, cw = byte0 // 8, len(img) // 8, C // 8
+    c_first, c_end = g0 // cw, (g0 + nw + cw - 1) // cw if nw else g0 // cw
+
+    def run(ca, cb):
+        wa, wb = max(g0, ca * cw), min(g0 + nw, cb * cw)
+        if wb > wa:
+            lib().orc_jf64_accumulate(_ptr(img) + 8 * (wa - g0), wa, wb - wa, cw, _ptr(d))
+
+    parts = [(c_first + a, c_first + b) for a, b in _parts(c_end - c_first, threads)]
+    _run_parts(run, parts)
     return d
 
 

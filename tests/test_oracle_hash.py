@@ -204,3 +204,21 @@ def test_root_chain():
         assert O.root(0x1234, e) != r
     e = d.copy(); e[[1, 2]] = e[[2, 1]]
     assert O.root(0x1234, e) != r
+
+
+def test_oracle_threads_agree():
+    """digests (and pack/unpack) are identical with 1 or
+    N oracle threads -- each thread owns whole chunks / whole tensors."""
+    from workloads import configs as W
+    g = W.random_table(77, 300, max_bytes=9000)
+    for C in (4096, 1 << 16):
+        lay = O.layout_of_group(g, C)
+        ts = O.gen_group(g, 3)
+        img1 = O.pack(ts, lay)
+        for th in (2, 3, 8, 1000):
+            assert np.array_equal(O.pack(ts, lay, threads=th), img1)
+            for a, b in ((0, lay.L), (8 * 37, lay.L - 8 * 5), (C + 8, 3 * C + 16)):
+                assert np.array_equal(O.jf64(img1[a:b], C, a, lay.n_c, threads=th),
+                                      O.jf64(img1[a:b], C, a, lay.n_c)), (th, a, b)
+            for x, y in zip(O.unpack(img1, lay, threads=th), ts):
+                assert np.array_equal(x, y.view(np.uint8).reshape(-1))
