@@ -212,7 +212,7 @@ def oracle_step(lay, ts, threads: int = 1):
     return out
 
 
-def cpu_baseline(cfg_name: str, sample_bytes: int = 2 << 30, reps: int = 2):
+def cpu_baseline(cfg_name: str, sample_bytes: int = 2 << 30, reps: int = 8):
     """The oracle on the box's host cores (all of them), plus its 1-thread
     figure; bounded sample."""
     g2, lay, ts, total = oracle_sample(cfg_name, sample_bytes)
