@@ -379,7 +379,23 @@ typedef void (*jitc_hang_fn)(void* user, uint64_t tag, double waited_ms);
  * run fingerprint -> exchange -> select -> sharded capture -> commit among
  * themselves on their watchdog threads -- the paper's whole user-level
  * protocol with no Python and no scheduler. */
+/* The same action over an NCCL communicator (jitc_comm_init) needs the
+ * liveness table below: failed ranks are dropped with
+ * ncclCommShrink(NCCL_SHRINK_ABORT), and the exchange and the commit barrier
+ * run over the shrunk NCCL communicator.  Without either table the action
+ * returns JITC_ESTATE. */
 enum { JITC_ON_HANG_NOTIFY = 0, JITC_ON_HANG_LOCAL_CAPTURE = 1, JITC_ON_HANG_COLLECTIVE_CAPTURE = 2 };
+/* Liveness table for failure localisation with the NCCL transport
+ * (§3.1: the survivors must tell a dead peer from a hung
+ * one).  Maps <dir>/liveness -- a directory on /dev/shm shared by the ranks of
+ * ONE box, created on first use, 8 KiB -- and starts a thread that writes this
+ * rank's CLOCK_MONOTONIC heartbeat (slot = job rank cfg.rank, < 1024) every
+ * 10 ms until jitc_destroy.  A communicator member whose heartbeat is older
+ * than the watchdog timeout, or was never written, counts as dead, so every
+ * rank calls this before arming its watchdog.  Local; may be called again
+ * (re-maps).  Errors: JITC_EINVAL (null ctx/dir, rank out of range),
+ * JITC_EIO (file or mapping). */
+jitc_status jitc_liveness_init(jitc_ctx* ctx, const char* dir);
 jitc_status jitc_watch_event(jitc_ctx* ctx, void* event, uint64_t tag);
 jitc_status jitc_watchdog_start(jitc_ctx* ctx, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user);
 /* Blocks up to max_ms for the hang action to finish.  *fired = 1 if it did;

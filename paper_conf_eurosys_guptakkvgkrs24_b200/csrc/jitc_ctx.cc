@@ -126,6 +126,7 @@ void jitc_destroy(jitc_ctx* c) {
   for (ncclComm_t r : c->retired_comms) ncclCommAbort(r);
   c->retired_comms.clear();
   ipc_destroy(c);
+  liveness_destroy(c);
   for (auto& kv : c->groups) free_group(kv.second);
   for (int i = 0; i < jitc_ctx::kSlots; ++i) {
     if (c->ev_ready[i]) cudaEventDestroy(c->ev_ready[i]);

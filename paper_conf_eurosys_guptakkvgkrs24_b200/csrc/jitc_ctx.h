@@ -114,6 +114,20 @@ struct IpcComm {
   std::atomic<bool> hb_run{false};
 };
 
+// Liveness table for the NCCL transport (NEXT-1 failure localisation; the
+// IPC transport keeps its heartbeats in IpcCtl): one CLOCK_MONOTONIC
+// heartbeat per JOB rank in a small file on /dev/shm shared by the ranks of
+// one box, refreshed every 10 ms by a thread of each process
+// (jitc_liveness_init).
+constexpr int kLiveMaxRanks = 1024;
+struct Liveness {
+  std::string path;
+  uint64_t* hb = nullptr;  // kLiveMaxRanks heartbeats, indexed by job rank
+  size_t bytes = 0;
+  std::thread th;
+  std::atomic<bool> run{false};
+};
+
 }  // namespace jitc
 
 using namespace jitc;
@@ -156,6 +170,7 @@ struct jitc_ctx {
   int comm_n = 0, comm_rank = -1;
   std::vector<int32_t> comm_job;  // comm rank -> job rank
   std::unique_ptr<IpcComm> ipc;   // IPC transport (instead of `comm`)
+  std::unique_ptr<Liveness> live; // heartbeats for the NCCL transport (jitc_liveness_init)
   std::vector<uint8_t> aux;       // user CPU state for the next commit (jitc_set_aux)
   uint64_t* d_small = nullptr;    // 64 B device scratch for size exchange / barrier
   uint32_t* d_work = nullptr;     // K1/K2/K3 batch counters (self-resetting)
@@ -402,6 +417,9 @@ jitc_status ipc_post(jitc_ctx* c, uint64_t* counter, uint64_t value, cudaStream_
 jitc_status ipc_wait(const uint64_t* counter, uint64_t value, const char* what);
 // job ranks of the communicator whose heartbeat is older than stale_ms (dead processes)
 std::vector<int32_t> ipc_stale_ranks(jitc_ctx* c, double stale_ms);
+// the same for whichever table this ctx has (IPC control block or liveness file)
+std::vector<int32_t> stale_ranks(jitc_ctx* c, double stale_ms);
+void liveness_destroy(jitc_ctx* c);
 void ipc_destroy(jitc_ctx* c);
 uint32_t group_slot(const jitc_ctx* c, uint32_t group);
 

@@ -126,6 +126,28 @@ std::vector<int32_t> ipc_stale_ranks(jitc_ctx* c, double stale_ms) {
   return out;
 }
 
+std::vector<int32_t> stale_ranks(jitc_ctx* c, double stale_ms) {
+  if (c->ipc) return ipc_stale_ranks(c, stale_ms);
+  std::vector<int32_t> out;
+  if (!c->live) return out;
+  const uint64_t now = mono_us();
+  for (int q = 0; q < c->comm_n; ++q) {
+    const int32_t j = c->comm_job[q];
+    if (q == c->comm_rank) continue;
+    uint64_t hb = (j >= 0 && j < kLiveMaxRanks) ? load_acq(&c->live->hb[j]) : 0;
+    if (hb == 0 || now > hb + (uint64_t)(stale_ms * 1000.0)) out.push_back(j);
+  }
+  return out;
+}
+
+void liveness_destroy(jitc_ctx* c) {
+  if (!c->live) return;
+  c->live->run = false;
+  if (c->live->th.joinable()) c->live->th.join();
+  if (c->live->hb) munmap(c->live->hb, c->live->bytes);
+  c->live.reset();
+}
+
 void ipc_destroy(jitc_ctx* c) {
   if (!c->ipc) return;
   IpcComm& ic = *c->ipc;
@@ -225,4 +247,38 @@ extern "C" jitc_status jitc_comm_init_ipc(jitc_ctx* c, const char* comm_dir, int
   });
   c->ipc = std::move(ic);
   return ipc_barrier(c);
+}
+
+// Liveness table for the NCCL transport (see include/jitc.h).
+extern "C" jitc_status jitc_liveness_init(jitc_ctx* c, const char* dir) {
+  if (!c || !dir) return fail(JITC_EINVAL, "jitc_liveness_init: null argument");
+  if (c->cfg.rank < 0 || c->cfg.rank >= kLiveMaxRanks)
+    return fail(JITC_EINVAL, "jitc_liveness_init: job rank out of range [0, " + std::to_string(kLiveMaxRanks) + ")");
+  liveness_destroy(c);
+  std::unique_ptr<Liveness> lv(new Liveness());
+  mkdir(dir, 0700);
+  lv->path = std::string(dir) + "/liveness";
+  lv->bytes = align_up(sizeof(uint64_t) * kLiveMaxRanks, 4096);
+  int fd = open(lv->path.c_str(), O_RDWR | O_CREAT, 0600);
+  if (fd < 0) return fail(JITC_EIO, "jitc_liveness_init: open " + lv->path + ": " + strerror(errno));
+  flock(fd, LOCK_EX);
+  struct stat sb;
+  bool ok = fstat(fd, &sb) == 0 && ((uint64_t)sb.st_size >= lv->bytes || ftruncate(fd, (off_t)lv->bytes) == 0);
+  void* p = ok ? mmap(nullptr, lv->bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0) : MAP_FAILED;
+  flock(fd, LOCK_UN);
+  close(fd);
+  if (p == MAP_FAILED) return fail(JITC_EIO, "jitc_liveness_init: mapping " + lv->path);
+  lv->hb = static_cast<uint64_t*>(p);
+  const int32_t me = c->cfg.rank;
+  store_rel(&lv->hb[me], mono_us());
+  lv->run = true;
+  Liveness* l = lv.get();
+  lv->th = std::thread([l, me] {
+    while (l->run) {
+      store_rel(&l->hb[me], mono_us());
+      std::this_thread::sleep_for(std::chrono::milliseconds(10));
+    }
+  });
+  c->live = std::move(lv);
+  return JITC_OK;
 }

@@ -13,20 +13,17 @@ using namespace jitc;
 // GIL cannot block it) on the library's non-blocking streams.
 
 // The paper's user-level protocol run by the survivors themselves
-// (PAPER.md:105-116): peers whose heartbeat went stale are dead; drop them
+// (PAPER.md:105-116): peers whose heartbeat went stale are dead (IPC control
+// block, or the liveness table of jitc_liveness_init for NCCL); drop them
 // from the communicator (ncclCommShrink(ABORT), which also aborts the hung
 // collective, or an IPC shrink), then fingerprint -> exchange -> select ->
 // sharded capture -> commit among the survivors, all on this thread.
 static jitc_status collective_capture(jitc_ctx* c, jitc_stats* st) {
-  std::vector<int32_t> failed;
-  if (c->ipc) {
-    failed = ipc_stale_ranks(c, c->timeout_ms);
-  } else if (!c->comm) {
-    return local_capture(c, st);
-  } else {
-    return fail(JITC_ESTATE, "collective capture needs failure localisation: use the IPC transport "
-                             "(heartbeats) or JITC_ON_HANG_NOTIFY and shrink from the harness");
-  }
+  if (!has_comm(c)) return local_capture(c, st);
+  if (!c->ipc && !c->live)
+    return fail(JITC_ESTATE, "collective capture needs failure localisation: use the IPC transport, "
+                             "jitc_liveness_init (NCCL transport), or JITC_ON_HANG_NOTIFY and shrink from the harness");
+  std::vector<int32_t> failed = stale_ranks(c, c->timeout_ms);
   jitc_status r = JITC_OK;
   if (!failed.empty()) {
     r = jitc_comm_shrink(c, failed.data(), (int32_t)failed.size());

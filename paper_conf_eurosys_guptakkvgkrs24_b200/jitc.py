@@ -94,6 +94,7 @@ def lib() -> ctypes.CDLL:
         "jitc_comm_shrink": ([vp, P(i32), i32], i32),
         "jitc_comm_destroy": ([vp], i32),
         "jitc_comm_init_ipc": ([vp, ctypes.c_char_p, i32, i32, P(i32)], i32),
+        "jitc_liveness_init": ([vp, ctypes.c_char_p], i32),
         "jitc_fingerprint": ([vp, u32, vp, sz, P(sz)], i32),
         "jitc_exchange_records": ([vp, vp, sz, vp, sz, P(sz)], i32),
         "jitc_select_consistent_replica": ([vp, sz, P(i32), i32, vp, sz, P(sz)], i32),
@@ -145,7 +146,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
             "jitc_inject_release", "jitc_capture_local", "jitc_set_aux", "jitc_get_aux", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop", "jitc_watchdog_failed", "jitc_capture_plan", "jitc_capture_fanout",
-            "jitc_attach_image"]
+            "jitc_attach_image", "jitc_liveness_init"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE, ON_HANG_COLLECTIVE_CAPTURE = 0, 1, 2
 
 
@@ -362,6 +363,11 @@ class Context:
         """Intra-node communicator over CUDA IPC + shared memory (no NCCL)."""
         jr = _i32arr(list(job_ranks)) if job_ranks is not None else None
         _check(self._L.jitc_comm_init_ipc(self._h, comm_dir.encode(), nranks, comm_rank, jr), "jitc_comm_init_ipc")
+
+    def liveness_init(self, live_dir: str):
+        """Heartbeat table for failure localisation over an NCCL communicator
+        (lets ON_HANG_COLLECTIVE_CAPTURE run with jitc_comm_init)."""
+        _check(self._L.jitc_liveness_init(self._h, live_dir.encode()), "jitc_liveness_init")
 
     def comm_shrink(self, failed: Sequence[int]):
         _check(self._L.jitc_comm_shrink(self._h, _i32arr(list(failed)), len(failed)), "jitc_comm_shrink")
