@@ -207,6 +207,48 @@ def test_corrupt_host_image_exact_chunk(J, shm):
     ctx.restore(g.group, J.HOST)
 
 
+def test_fuzzed_manifest_and_commit_record_refused(J, shm):
+    """Robustness of the metadata path (PAPER.md:136, :140 -- a checkpoint
+    whose metadata is incomplete or corrupted is discarded): 300 random
+    single-byte changes and truncations of the committed manifest and commit
+    record.  Every one must be refused with EINCOMPLETE or ELAYOUT -- never
+    accepted, never a crash -- and the intact files then restore bit-exact."""
+    g = _small_groups()[3]
+    C = 4096
+    st = _state(g, 6)
+    ctx = _ctx(J, C, image_dir=shm)
+    ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+    _pipeline(J, ctx)
+    paths = {k: f"{shm}/g{g.group}.{k}" for k in ("manifest", "commit")}
+    orig = {k: open(p, "rb").read() for k, p in paths.items()}
+    rng = np.random.default_rng(11)
+    seen = set()
+    for it in range(300):
+        which = "manifest" if it % 3 else "commit"
+        b = bytearray(orig[which])
+        if it % 10 == 9:
+            b = b[:int(rng.integers(0, len(b)))]                 # torn write
+        else:
+            pos = int(rng.integers(0, len(b)))
+            b[pos] ^= int(rng.integers(1, 256))                  # any change to one byte
+        with open(paths[which], "wb") as f:
+            f.write(bytes(b))
+        with pytest.raises(J.JitcError) as e:
+            ctx.restore(g.group, J.HOST)
+        assert e.value.status in (J.EINCOMPLETE, J.ELAYOUT), (which, it, e.value)
+        seen.add(e.value.status)
+        with open(paths[which], "wb") as f:
+            f.write(orig[which])
+    assert J.EINCOMPLETE in seen
+    st.scramble()
+    ctx.restore(g.group, J.HOST)
+    ctx.verify(g.group)
+    torch.cuda.synchronize()
+    for i, t in enumerate(g.tensors):
+        assert np.array_equal(st.tensor_bytes(i).cpu().numpy(), O.gen_tensor_bytes(t, 6, g.group)), t.name
+    ctx.close()
+
+
 def test_uncommitted_refused(J, shm):
     g = W.random_table(4, 10)
     st = _state(g, 6)
