@@ -91,7 +91,7 @@ class ClockSampler:
 def calibrate_links(device: int, world: int, nccl_group=None, host_gib: int = 2):
     """In-run link calibration, untimed, before the
     timed region: B_d2h / B_h2d with every rank copying at once (64 MiB
-    cudaMemcpyAsync pieces of pinned memory, best of 3), B_hbm from a 4 GiB
+    cudaMemcpyAsync pieces of pinned memory, best of 5), B_hbm from a 4 GiB
     device-to-device copy (read + write bytes), B_nvl from a 256 MiB-per-rank
     NCCL all-gather (bus bandwidth (n-1)/n * total / t) when an NCCL group is
     given.  Returns GB/s (per rank for the host link)."""
@@ -104,7 +104,7 @@ def calibrate_links(device: int, world: int, nccl_group=None, host_gib: int = 2)
     s = torch.cuda.Stream(device)
     out = {}
 
-    def timed(fn, reps=3):
+    def timed(fn, reps=5):
         best = None
         for _ in range(reps):
             if world > 1:
@@ -141,9 +141,49 @@ def calibrate_links(device: int, world: int, nccl_group=None, host_gib: int = 2)
         t = timed(lambda: dist.all_gather_into_tensor(allb, blk, group=nccl_group))
         out["nvl_allgather_busbw_GBps"] = round((world - 1) * blk.numel() / t / 1e9, 1)
     torch.cuda.empty_cache()
-    out["how"] = (f"{host_gib} GiB pinned, 64 MiB pieces, all {world} rank(s) at once, best of 3; "
+    out["how"] = (f"{host_gib} GiB pinned, 64 MiB pieces, all {world} rank(s) at once, best of 5, after the warm-up steps; "
                   "HBM: 4 GiB D2D copy (read+write)")
     return out
+
+
+def per_tensor_d2h(states, device: int, world: int, buf_gib: int = 4, reps: int = 2):
+    """the CE-only "pure copy" baseline -- every registered
+    tensor copied D2H on its own (one cudaMemcpyAsync per tensor, like a
+    per-tensor torch.save), with no fingerprint and no staging.  Destinations
+    wrap around a pinned buffer of buf_gib GiB at 256-B-aligned offsets (the
+    link, not the host footprint, is what is measured).  Every rank copies its
+    FULL state at once (the paper's every-rank-saves protocol at raw copy
+    speed).  Untimed region; CUDA events on the copy stream, best of reps."""
+    import torch
+    import torch.distributed as dist
+    tensors = [st.tensor_bytes(i) for st in states.values() for i in range(len(st.spec.tensors))]
+    total = sum(t.numel() for t in tensors)
+    h = torch.empty(buf_gib << 30, dtype=torch.uint8, pin_memory=True)
+    s = torch.cuda.Stream(device)
+    best = None
+    for _ in range(reps):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(s):
+            e0.record(s)
+            pos = 0
+            for t in tensors:
+                n = t.numel()
+                if pos + n > h.numel():
+                    pos = 0
+                h[pos:pos + n].copy_(t, non_blocking=True)
+                pos += (n + 255) // 256 * 256
+            e1.record(s)
+        e1.synchronize()
+        ms = e0.elapsed_time(e1)
+        best = ms if best is None else min(best, ms)
+    del h
+    return {"tensors": len(tensors), "bytes": total, "ms": round(best, 2),
+            "GBps": round(total / (best * 1e-3) / 1e9, 2),
+            "how": "one cudaMemcpyAsync D2H per registered tensor into pinned memory (no digest, no staging); "
+                   "all ranks at once; CUDA events, best of %d" % reps}
 
 
 def host_link_roofline(L_total, world, capture_ms, restore_ms, links):
@@ -320,7 +360,6 @@ def run_jitc(args):
     nccl_group = None
     if world > 1 and not os.environ.get("JITC_BENCH_SHARE_GPU"):
         nccl_group = dist.new_group(backend="nccl")
-    links = calibrate_links(local, world, nccl_group) if not args.no_calibrate else None
 
     healthy = list(range(world))
     per = {"fingerprint": [], "select": [], "capture": [], "commit": [], "restore": [], "verify": []}
@@ -353,6 +392,11 @@ def run_jitc(args):
 
     for _ in range(args.warmup):
         step(False)
+    # link calibration after the warm-up steps, when the host image's pages and
+    # the pinned buffers are settled (one box read 41 GB/s D2H right after
+    # registering 25 GB, 56 GB/s later); still outside the timed region
+    links = calibrate_links(local, world, nccl_group) if not args.no_calibrate else None
+    f3 = per_tensor_d2h(states, local, world) if not args.no_calibrate else None
     ctx.reset_counters()
     if world > 1:
         dist.barrier()
@@ -513,6 +557,7 @@ def run_jitc(args):
             "capture_GBps": round(L_total / world / (cap_ms * 1e-3) / 1e9, 3),
             "restore_GBps": round(L_total / (res_ms * 1e-3) / 1e9, 3),
             "host_link_roofline": host_link_roofline(L_total, world, med["capture"], res_ms, links),
+            "per_tensor_d2h_baseline": f3,
             "roofline": {"kernel": kinds[dom], "bound": "hbm", "achieved": round(achieved, 1) if achieved else None,
                          "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
                          "traffic": traffic, "peak_source": peak_src,
