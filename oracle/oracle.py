@@ -563,7 +563,10 @@ def manifest_trailer(body: bytes) -> int:
     return fold_fmix64(np.frombuffer(pad, dtype="<u8").tolist())
 
 
-def encode_manifest(gs: GroupSel, v_star: int, lay: Layout, d: np.ndarray) -> bytes:
+def encode_manifest(gs: GroupSel, v_star: int, lay: Layout, d: np.ndarray, aux: bytes = b"") -> bytes:
+    """O4b, plus the aux section of DESIGN.md §5 (the user's opaque CPU state,
+    PAPER.md:132: u64 aux_len, the bytes, zero padding to 8) after the shard
+    table; the trailer covers every preceding byte."""
     k = len(gs.writers)
     h = struct.pack("<IHHIIQQQQQII", MAGIC_M, 1, 0, gs.group, len(lay.names), v_star,
                     lay.layout_hash, lay.C, lay.n_c, lay.L, k, 0)
@@ -578,7 +581,8 @@ def encode_manifest(gs: GroupSel, v_star: int, lay: Layout, d: np.ndarray) -> by
     for s, w in enumerate(gs.writers):
         c0, c1 = shard(lay.n_c, k, s)
         st += struct.pack("<iIQQ", w, 0, c0, c1)
-    body = h + tt + dd + st
+    ax = struct.pack("<Q", len(aux)) + bytes(aux) + b"\0" * ((-len(aux)) % 8)
+    body = h + tt + dd + st + ax
     return body + struct.pack("<Q", manifest_trailer(body))
 
 
@@ -623,9 +627,13 @@ def decode_manifest(man: bytes):
         dts.append(dt); nbs.append(nb); offs.append(off)
     p += (-(p - p0)) % 8
     d = np.frombuffer(man, dtype="<u8", count=n_c, offset=p).astype(np.uint64); p += 8 * n_c
-    (rt,) = struct.unpack_from("<Q", man, p)
+    (rt,) = struct.unpack_from("<Q", man, p); p += 8
+    shards = [struct.unpack_from("<iIQQ", man, p + 24 * s) for s in range(k)]; p += 24 * k
+    (aux_len,) = struct.unpack_from("<Q", man, p); p += 8
+    aux = man[p:p + aux_len]
     lay = Layout(names, nbs, dts, offs, L, C, lh)
-    return dict(group=group, v_star=v_star, layout=lay, d=d, root=rt, writers=writers)
+    return dict(group=group, v_star=v_star, layout=lay, d=d, root=rt, writers=writers,
+                shards=[(w, c0, c1) for w, _, c0, c1 in shards], aux=aux)
 
 
 def restore_sim(host: np.ndarray, man: Optional[bytes], commit: Optional[bytes]):

@@ -159,6 +159,39 @@ def test_c5_tp4_dp2_sharded_capture_and_replacement(J, shm):
     job.close()
 
 
+def test_manifest_and_commit_record_bytes_equal_oracle(J, shm):
+    """A8 parity (byte work => bit-exact): the manifest and commit record the
+    library writes for every C5 group -- k = 2 writers, a lone writer after
+    rank 5 died, the user's CPU-state aux bytes -- equal the
+    oracle's O4b encoding of the oracle's own selection,
+    layout and digests, byte for byte."""
+    w = _small(W.c5(n_layer=2))
+    job = Job(J, w, shm, dead=(5,))
+    aux = b"iteration=40;rng=" + bytes(range(29))
+    for c in job.ctx.values():
+        c.set_aux(aux)
+    healthy = sorted(job.ctx)
+    blobs = b"".join(job.ctx[r].fingerprint() for r in healthy)
+    ref = O.select(blobs, healthy)
+    st, sel, got = job.select()
+    assert st == 0
+    job.capture_commit(sel)
+    n_checked = 0
+    for gs in ref.groups:
+        if not gs.writers:
+            continue
+        g = next(x for x in w.groups if x.group == gs.group)
+        lay = O.layout_of_group(g, C)
+        d = O.jf64(O.pack(_expected(g, w.seed, []), lay), C, 0, lay.n_c)
+        want_man = O.encode_manifest(gs, ref.v_star, lay, d, aux)
+        got_man = open(f"{shm}/g{gs.group}.manifest", "rb").read()
+        assert got_man == want_man, gs.group
+        assert open(f"{shm}/g{gs.group}.commit", "rb").read() == O.commit_record(gs.group, ref.v_star, want_man)
+        n_checked += 1
+    assert n_checked == len(w.groups)
+    job.close()
+
+
 def test_c5_bitflip_conflict_and_image_corruption(J, shm):
     """C5 injections: a flip in rank 2's master (HBM) makes partition 2 a 1-1
     tie (ECONFLICT, the flipped chunk listed); after a clean capture, a flip

@@ -90,3 +90,30 @@ def test_half_step_detected():
         assert (O.root(lay.layout_hash, d0) != O.root(lay.layout_hash, d1)) == bool(touched), split
         n_split += 1
     assert n_split == len(ts) - 1
+
+
+def test_manifest_roundtrip_aux_and_every_byte_covered():
+    """O4b + the aux section (PAPER.md:132 CPU state carried
+    opaque; PAPER.md:136 metadata last): decode(encode(x)) == x, the shard
+    table is O5's, and changing ANY single byte of the manifest body is caught
+    by the trailer (fold_fmix64 is a chain of bijections over LE words, so a
+    change confined to one word always changes it) -> EINCOMPLETE."""
+    g = W.random_table(5, 7, max_bytes=3000)
+    lay = O.layout_of_group(g, 4096)
+    img = O.pack(O.gen_group(g, 2), lay)
+    d = O.jf64(img, lay.C, 0, lay.n_c)
+    gs = O.GroupSel(0, O.REQUIRED, writers=[1, 4, 6])
+    for aux in (b"", b"x", b"iteration=17;rng=" + bytes(range(40))):
+        man = O.encode_manifest(gs, 9, lay, d, aux)
+        assert len(man) % 8 == 0
+        m = O.decode_manifest(man)
+        assert m["aux"] == aux and m["writers"] == [1, 4, 6] and m["v_star"] == 9
+        assert np.array_equal(m["d"], d) and m["root"] == O.root(lay.layout_hash, d)
+        assert m["shards"] == [(w, *O.shard(lay.n_c, 3, s)) for s, w in enumerate([1, 4, 6])]
+        assert m["layout"].offsets == lay.offsets and m["layout"].names == lay.names
+        com = O.commit_record(0, 9, man)
+        assert O.restore_sim(img, man, com)[0] == O.OK
+    for pos in range(len(man) - 8):
+        bad = bytearray(man)
+        bad[pos] ^= 0x5A
+        assert O.restore_sim(img, bytes(bad), com)[0] == O.EINCOMPLETE, pos
