@@ -192,6 +192,35 @@ def test_manifest_and_commit_record_bytes_equal_oracle(J, shm):
     job.close()
 
 
+def test_fingerprint_blobs_bytes_equal_oracle(J, shm):
+    """A3/A4 parity: every rank's fingerprint blob -- header, job topology
+    (including groups it only declares) and one O4 record per held group with
+    the K1 digests and root -- equals the oracle's encoding of the oracle's
+    layout, digests and phase word, byte for byte (C5, TP4 x DP2, 8 ranks;
+    one rank DIRTY at the next version to cover the phase/version fields)."""
+    w = _small(W.c5(n_layer=2))
+    job = Job(J, w, shm)
+    job.ctx[3].mark(3, V + 1, J.DIRTY)
+    torch.cuda.synchronize()
+    topo = [O.TopoEntry(g.group, g.policy, list(g.members)) for g in w.groups]
+    digests = {}
+    for g in w.groups:
+        lay = O.layout_of_group(g, C)
+        d = O.jf64(O.pack(_expected(g, w.seed, []), lay), C, 0, lay.n_c)
+        digests[g.group] = (lay, d)
+    for r in sorted(job.ctx):
+        recs = []
+        for g in w.groups:
+            if r not in g.members:
+                continue
+            lay, d = digests[g.group]
+            version, phase = (V + 1, O.DIRTY) if (r, g.group) == (3, 3) else (V, O.CLEAN)
+            recs.append(O.Record(r, g.group, g.policy, phase, version, lay.layout_hash, C, lay.L, d,
+                                 O.root(lay.layout_hash, d)))
+        assert job.ctx[r].fingerprint() == O.encode_blob(r, topo, recs), r
+    job.close()
+
+
 def test_c5_bitflip_conflict_and_image_corruption(J, shm):
     """C5 injections: a flip in rank 2's master (HBM) makes partition 2 a 1-1
     tie (ECONFLICT, the flipped chunk listed); after a clean capture, a flip
