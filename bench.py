@@ -231,6 +231,16 @@ def oracle_sample(cfg_name: str, sample_bytes: int):
     return g2, lay, ts, total
 
 
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def host_threads() -> int:
     try:
         return len(os.sched_getaffinity(0))
@@ -268,7 +278,7 @@ def cpu_baseline(cfg_name: str, sample_bytes: int = 2 << 30, reps: int = 8):
     return {"value": round(lay.L / dt / 1e9, 4), "unit": "GB/s", "cores": nth, "kind": "oracle",
             "sample": f"first {lay.L / 2**30:.2f} GiB of the {cfg_name} REQUIRED-group image "
                       f"({len(lay.names)} tensors), pack+JF64+JF64+unpack, {reps} reps, {nth} threads",
-            "seconds_per_sample": round(dt, 3),
+            "seconds_per_sample": round(dt, 3), "cpu_model": cpu_model(), "nproc": os.cpu_count(),
             "single_thread": {"value": round(lay.L / out[1] / 1e9, 4), "cores": 1,
                               "seconds_per_sample": round(out[1], 3)}}
 
@@ -294,6 +304,7 @@ def run_reference(args):
             "config": {"workload": W.CONFIGS[args.config]().name, "sample_bytes": lay.L,
                        "note": "bounded prefix of the same workload's REQUIRED image; oracle pack+JF64+JF64+unpack"},
             "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": nth, "kind": "oracle",
+                             "cpu_model": cpu_model(),
                              "sample": f"first {lay.L / 2**20:.0f} MiB of the {args.config} REQUIRED-group image, "
                                        f"{nth} threads"},
             "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
