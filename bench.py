@@ -449,6 +449,41 @@ def run_jitc(args):
                           "sharded_capture_s": round(statistics.median(per["capture"]) * 1e-3, 4),
                           "sharded_host_link_bytes_total": L_total}
 
+    # PEER restore (SURVEY.md §8(d) d.5 "PEER restore"; PAPER.md:174, :184 copy
+    # from a replica): the last rank plays the replacement.  The selection is
+    # taken over the other ranks' records, its state is overwritten, and every
+    # rank calls jitc_restore(PEER): the k = n-1 writers pack their O5 ranges
+    # from live HBM and send them over the communicator (NVLink on a multi-GPU
+    # box), the replacement unpacks + verifies.  Max over ranks, host wall clock.
+    peer_restore = None
+    if world > 1 and not args.no_peer_restore:
+        victim = world - 1
+        blob = ctx.fingerprint()
+        allb = ctx.exchange_records(blob)
+        st_p, sel_p = J.select_consistent_replica(allb, list(range(world - 1)))
+        if st_p != J.OK:
+            raise RuntimeError(f"peer select: {J.parse_selection(sel_p)}")
+        if rank == victim:
+            for st in states.values():
+                st.scramble()
+        torch.cuda.synchronize()
+        dist.barrier()
+        t0 = time.perf_counter()
+        res_p = ctx.restore(J.ALL_GROUPS, J.PEER, sel_p)
+        if rank == victim:
+            for gid in states:
+                ctx.verify(gid)
+        dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64)
+        dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+        pb = torch.tensor([res_p["p2p_bytes"] if rank == victim else 0], dtype=torch.float64)
+        dist.all_reduce(pb, op=dist.ReduceOp.MAX)
+        peer_restore = {"replacement": victim, "writers": world - 1, "s": round(dt.item(), 4),
+                        "GBps": round(L_total / dt.item() / 1e9, 3), "replacement_ingress_bytes": int(pb.item()),
+                        "transport": args.transport,
+                        "how": "selection over ranks 0..n-2; the replacement's tensors overwritten first; "
+                               "jitc_restore(PEER) on every rank + jitc_verify on the replacement; host wall clock, "
+                               "max over ranks"}
+
     # robustness variant: one more step while an emulated
     # hung collective (32 spinning CTAs on another stream) occupies the GPU,
     # as when a NCCL kernel waits forever on a dead peer
@@ -588,6 +623,7 @@ def run_jitc(args):
             "gpu_launches": launches[0],
             "under_hang": under_hang,
             "paper_protocol": paper_protocol,
+            "peer_restore": peer_restore,
             "comm_rebuild": comm_rebuild,
             "watchdog_on_hang": on_hang,
             "clocks": clk.summary(),
@@ -623,6 +659,7 @@ def main():
     ap.add_argument("--no-watchdog", action="store_true", help="N = 1: skip the watchdog on-hang capture variant")
     ap.add_argument("--watchdog-ms", type=int, default=200, help="watchdog hang timeout for that variant")
     ap.add_argument("--no-comm-rebuild", action="store_true", help="N > 1: skip timing shrink + re-init")
+    ap.add_argument("--no-peer-restore", action="store_true", help="N > 1: skip the PEER-restore variant")
     ap.add_argument("--no-calibrate", action="store_true", help="skip the in-run host-link / HBM / NVLink calibration")
     ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],

@@ -129,7 +129,7 @@ typedef struct {
     double ms_device;          /* CUDA-event span of the call on the library streams           */
     double ms_kernel;          /* sum of the call's kernel durations (needs JITC_F_TIME_KERNELS)*/
     uint64_t image_bytes;      /* image bytes this rank packed / unpacked / digested           */
-    uint64_t d2h_bytes, h2d_bytes, p2p_bytes;
+    uint64_t d2h_bytes, h2d_bytes, p2p_bytes;  /* p2p: bytes this rank received from peers (NCCL: plus sent) */
     uint64_t kernel_launches;  /* launches of this library's kernels during the call           */
     uint32_t rounds;           /* pipeline rounds                                              */
     int32_t first_bad_chunk;   /* ECORRUPT: first chunk whose digest mismatched, else -1       */

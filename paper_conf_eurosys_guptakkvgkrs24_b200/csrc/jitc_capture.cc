@@ -203,7 +203,7 @@ static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection
           const PlanOp& op = ops[q];
           if (op.kind == kOpSend) NC(ncclSend(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
           if (op.kind == kOpRecv) NC(ncclRecv(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
-          if (stats) stats->p2p_bytes += op.bytes;
+          if (stats && (op.kind == kOpSend || op.kind == kOpRecv)) stats->p2p_bytes += op.bytes;
         }
         NC(ncclGroupEnd());
       }

@@ -156,7 +156,7 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
           const PlanOp& op = ops[q];
           if (op.kind == kOpSend) NC(ncclSend(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
           if (op.kind == kOpRecv) NC(ncclRecv(c->staging + op.off, op.bytes, ncclUint8, op.peer, c->comm, c->s_comp));
-          if (stats) stats->p2p_bytes += op.bytes;
+          if (stats && (op.kind == kOpSend || op.kind == kOpRecv)) stats->p2p_bytes += op.bytes;
         }
         NC(ncclGroupEnd());
       }
