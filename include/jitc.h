@@ -73,7 +73,10 @@ enum {
     JITC_EUNSTABLE = -10,      /* bytes changed between fingerprint and capture          */
     JITC_ECORRUPT = -11,       /* restored bytes do not match the manifest digests       */
     JITC_EINCOMPLETE = -12,    /* checkpoint not committed (PAPER.md:136 metadata last)  */
-    JITC_EIO = -13             /* file / shm error                                       */
+    JITC_EIO = -13,            /* file / shm error                                       */
+    JITC_EPEER = -14           /* a communicator peer died while this call waited on it
+                                  (IPC transport: its heartbeat went stale); see
+                                  jitc_comm_dead, then jitc_comm_shrink and retry          */
 };
 
 /* Optimizer-step phase of a group, written by jitc_mark (PAPER.md:188 hooks). */
@@ -396,6 +399,14 @@ enum { JITC_ON_HANG_NOTIFY = 0, JITC_ON_HANG_LOCAL_CAPTURE = 1, JITC_ON_HANG_COL
  * (re-maps).  Errors: JITC_EINVAL (null ctx/dir, rank out of range),
  * JITC_EIO (file or mapping). */
 jitc_status jitc_liveness_init(jitc_ctx* ctx, const char* dir);
+/* Job ranks of the current communicator whose heartbeat (IPC control block,
+ * or the liveness table) is older than the dead-peer threshold: 2000 ms, or
+ * JITC_PEER_DEAD_MS read at communicator init.  Writes up to cap ranks and
+ * *n = count.  Local.  The recovery for reading R9 (a writer dies during the
+ * capture): a collective call returns JITC_EPEER, every survivor calls this,
+ * jitc_comm_shrink(dead), and re-runs fingerprint -> exchange -> select ->
+ * capture -> commit with k - 1 writers (HBM still holds the state). */
+jitc_status jitc_comm_dead(jitc_ctx* ctx, int32_t* ranks, int32_t cap, int32_t* n);
 jitc_status jitc_watch_event(jitc_ctx* ctx, void* event, uint64_t tag);
 jitc_status jitc_watchdog_start(jitc_ctx* ctx, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user);
 /* Blocks up to max_ms for the hang action to finish.  *fired = 1 if it did;

@@ -161,7 +161,7 @@ static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection
     // IPC: my readers must have consumed the round that last used this slot
     if (ic && packs && j >= S)
       for (int r : readers) {
-        jitc_status st = ipc_wait(&ic->ctl->cap_consumed[ic->slot[r]][gsl], seq - S, "a mover to consume a round");
+        jitc_status st = ipc_wait_peer(*ic, r, &ic->ctl->cap_consumed[ic->slot[r]][gsl], seq - S, "a mover to consume a round");
         if (st) return st;
       }
     // 1. K2: pack my block (re-digest into d_dig2)
@@ -184,7 +184,7 @@ static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection
         const PlanOp& op = ops[q];
         if (op.kind != kOpRecv) continue;
         recv = true;
-        jitc_status st = ipc_wait(&ic->ctl->cap_posted[ic->slot[op.peer]][gsl], seq, "a writer to post a round");
+        jitc_status st = ipc_wait_peer(*ic, op.peer, &ic->ctl->cap_posted[ic->slot[op.peer]][gsl], seq, "a writer to post a round");
         if (st) return st;
         CU(cudaMemcpyAsync(c->staging + op.off, ic->peer_staging[op.peer] + op.off, op.bytes, cudaMemcpyDefault,
                            c->s_comp));
@@ -230,7 +230,7 @@ static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection
   // IPC: my staging may be reused once this call returns -- wait for my readers
   if (ic && !readers.empty())
     for (int r : readers) {
-      jitc_status st = ipc_wait(&ic->ctl->cap_consumed[ic->slot[r]][gsl], (gen << 24) | J, "a mover to finish");
+      jitc_status st = ipc_wait_peer(*ic, r, &ic->ctl->cap_consumed[ic->slot[r]][gsl], (gen << 24) | J, "a mover to finish");
       if (st) return st;
     }
   if (stats) stats->rounds += rounds;

@@ -112,6 +112,7 @@ struct IpcComm {
   std::map<uint32_t, uint64_t> digest_gen;  // PEER digest hand-offs per group slot
   std::thread hb_thread;                    // heartbeat writer (failure localisation, NEXT-1)
   std::atomic<bool> hb_run{false};
+  double dead_ms = 2000.0;                  // a peer whose heartbeat is older is dead (JITC_PEER_DEAD_MS)
 };
 
 // Liveness table for the NCCL transport (NEXT-1 failure localisation; the
@@ -415,6 +416,10 @@ jitc_status ipc_barrier(jitc_ctx* c);
 jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len);
 jitc_status ipc_post(jitc_ctx* c, uint64_t* counter, uint64_t value, cudaStream_t s);
 jitc_status ipc_wait(const uint64_t* counter, uint64_t value, const char* what);
+// the same, failing with JITC_EPEER if comm rank `peer`'s heartbeat goes stale meanwhile
+jitc_status ipc_wait_peer(const IpcComm& ic, int peer, const uint64_t* counter, uint64_t value, const char* what);
+double peer_dead_ms();
+bool ipc_peer_dead(const IpcComm& ic, int peer);  // comm rank's heartbeat older than ic.dead_ms
 // job ranks of the communicator whose heartbeat is older than stale_ms (dead processes)
 std::vector<int32_t> ipc_stale_ranks(jitc_ctx* c, double stale_ms);
 // the same for whichever table this ctx has (IPC control block or liveness file)

@@ -41,6 +41,11 @@ inline void store_rel(uint64_t* p, uint64_t v) { __atomic_store_n(p, v, __ATOMIC
 
 constexpr double kIpcTimeoutMs = 600000.0;
 
+uint64_t mono_us() {
+  return (uint64_t)std::chrono::duration_cast<std::chrono::microseconds>(
+             std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
 }  // namespace
 
 namespace jitc {
@@ -65,6 +70,37 @@ jitc_status ipc_wait(const uint64_t* counter, uint64_t value, const char* what) 
   return JITC_OK;
 }
 
+double peer_dead_ms() {
+  const char* e = getenv("JITC_PEER_DEAD_MS");
+  double v = e ? atof(e) : 0.0;
+  return v > 0 ? v : 2000.0;
+}
+
+bool ipc_peer_dead(const IpcComm& ic, int peer) {
+  const uint64_t hb = load_acq(&ic.ctl->heartbeat[ic.slot[peer]]);
+  return hb && mono_us() > hb + (uint64_t)(ic.dead_ms * 1000.0);
+}
+
+// Waits on a counter that comm rank `peer` advances; a peer whose heartbeat
+// (refreshed every 10 ms by its heartbeat thread) is older than ic.dead_ms is
+// dead: the wait fails with JITC_EPEER instead of spinning until the 10-minute
+// timeout (reading R9: a writer that dies during the capture).
+jitc_status ipc_wait_peer(const IpcComm& ic, int peer, const uint64_t* counter, uint64_t value, const char* what) {
+  const double t0 = now_ms();
+  uint32_t spins = 0;
+  while (load_acq(counter) < value) {
+    if (++spins > 1000) sched_yield();
+    if ((spins & 0x3FF) == 0) {
+      if (ipc_peer_dead(ic, peer))
+        return fail(JITC_EPEER, std::string("IPC transport: comm rank ") + std::to_string(peer) +
+                                    " died (heartbeat stale) while waiting for " + what);
+      if (now_ms() - t0 > kIpcTimeoutMs)
+        return fail(JITC_ESTATE, std::string("IPC transport: timed out waiting for ") + what);
+    }
+  }
+  return JITC_OK;
+}
+
 jitc_status ipc_post(jitc_ctx* c, uint64_t* counter, uint64_t value, cudaStream_t s) {
   uint64_t* dev = reinterpret_cast<uint64_t*>(c->ipc->ctl_dev + ((uint8_t*)counter - (uint8_t*)c->ipc->ctl));
   if (c->write_value64 && c->write_value64((CUstream)s, (CUdeviceptr)dev, value, 0) == CUDA_SUCCESS) return JITC_OK;
@@ -77,7 +113,7 @@ jitc_status ipc_barrier(jitc_ctx* c) {
   const uint64_t gen = ++ic.barrier_gen;
   store_rel(&ic.ctl->arrive[ic.slot[c->comm_rank]], gen);
   for (int q = 0; q < c->comm_n; ++q) {
-    jitc_status st = ipc_wait(&ic.ctl->arrive[ic.slot[q]], gen, "a barrier");
+    jitc_status st = ipc_wait_peer(ic, q, &ic.ctl->arrive[ic.slot[q]], gen, "a barrier");
     if (st) return st;
   }
   return JITC_OK;
@@ -107,11 +143,6 @@ jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, s
   if (cap < out.size() || !all) return fail(JITC_EINVAL, "jitc_exchange_records: buffer too small");
   memcpy(all, out.data(), out.size());
   return JITC_OK;
-}
-
-static uint64_t mono_us() {
-  return (uint64_t)std::chrono::duration_cast<std::chrono::microseconds>(
-             std::chrono::steady_clock::now().time_since_epoch()).count();
 }
 
 std::vector<int32_t> ipc_stale_ranks(jitc_ctx* c, double stale_ms) {
@@ -178,6 +209,7 @@ extern "C" jitc_status jitc_comm_init_ipc(jitc_ctx* c, const char* comm_dir, int
   if (!range) return fail(JITC_ECUDA, "jitc_comm_init_ipc: cuMemGetAddressRange unavailable");
   std::unique_ptr<IpcComm> ic(new IpcComm());
   ic->dir = comm_dir;
+  ic->dead_ms = peer_dead_ms();
   mkdir(ic->dir.c_str(), 0700);
   std::string path = ic->dir + "/ctl";
   ic->ctl_bytes = align_up(sizeof(IpcCtl), 4096);
@@ -280,5 +312,15 @@ extern "C" jitc_status jitc_liveness_init(jitc_ctx* c, const char* dir) {
     }
   });
   c->live = std::move(lv);
+  return JITC_OK;
+}
+
+extern "C" jitc_status jitc_comm_dead(jitc_ctx* c, int32_t* ranks, int32_t cap, int32_t* n) {
+  if (!c || !n || (cap > 0 && !ranks)) return fail(JITC_EINVAL, "jitc_comm_dead: bad argument");
+  if (!has_comm(c)) return fail(JITC_ESTATE, "jitc_comm_dead: no communicator");
+  if (!c->ipc && !c->live) return fail(JITC_ESTATE, "jitc_comm_dead: no heartbeats (IPC transport or jitc_liveness_init)");
+  std::vector<int32_t> d = stale_ranks(c, c->ipc ? c->ipc->dead_ms : peer_dead_ms());
+  *n = (int32_t)d.size();
+  for (int32_t i = 0; i < *n && i < cap; ++i) ranks[i] = d[i];
   return JITC_OK;
 }

@@ -110,7 +110,7 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
     // 0. IPC: the readers of my slot must have consumed the round that used it last
     if (ic && writes_slot && j >= S)
       for (int r : readers) {
-        jitc_status st = ipc_wait(&ic->ctl->consumed[ic->slot[r]][gs], seq - S, "a peer to consume a round");
+        jitc_status st = ipc_wait_peer(*ic, r, &ic->ctl->consumed[ic->slot[r]][gs], seq - S, "a peer to consume a round");
         if (st) return st;
       }
     // 1. host -> device on the copy stream
@@ -143,7 +143,7 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
       for (size_t q = i; q < e; ++q) {
         const PlanOp& op = ops[q];
         if (op.kind != kOpUnpack || op.peer == c->comm_rank) continue;
-        st = ipc_wait(&ic->ctl->posted[ic->slot[op.peer]][gs], seq, "a peer to post a round");
+        st = ipc_wait_peer(*ic, op.peer, &ic->ctl->posted[ic->slot[op.peer]][gs], seq, "a peer to post a round");
         if (st) return st;
         if (stats) stats->p2p_bytes += op.b - op.a;
       }
@@ -204,7 +204,7 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
   if (ic) {
     // my staging may be reused as soon as this call returns: wait for its readers
     for (int r : readers) {
-      jitc_status st = ipc_wait(&ic->ctl->consumed[ic->slot[r]][gs], base_round + J, "a peer to finish reading");
+      jitc_status st = ipc_wait_peer(*ic, r, &ic->ctl->consumed[ic->slot[r]][gs], base_round + J, "a peer to finish reading");
       if (st) return st;
     }
     ic->rounds[gs] = base_round + J;
@@ -330,6 +330,8 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
       std::vector<uint8_t> b;
       const double t0 = now_ms();
       while (!read_file(path, &b) || b.size() != 8 * g.n_c) {
+        if (ipc_peer_dead(*c->ipc, in.writers[0]))
+          return fail(JITC_EPEER, "jitc_restore: the lowest writer died before handing over its digests");
         if (now_ms() - t0 > 600000.0) return fail(JITC_ESTATE, "jitc_restore: no digests from the writers");
         usleep(200);
       }

@@ -19,11 +19,11 @@ SO_PATH = os.environ.get("JITC_SO", os.path.join(_PKG, "libjitc.so"))
 
 OK, EINVAL, ESTATE, ENOMEM, ECUDA, ENCCL = 0, -1, -2, -3, -4, -5
 ELAYOUT, ENOREPLICA, ECONFLICT, ENOCONSISTENT = -6, -7, -8, -9
-EUNSTABLE, ECORRUPT, EINCOMPLETE, EIO = -10, -11, -12, -13
+EUNSTABLE, ECORRUPT, EINCOMPLETE, EIO, EPEER = -10, -11, -12, -13, -14
 STATUS_NAMES = {v: k for k, v in dict(
     OK=OK, EINVAL=EINVAL, ESTATE=ESTATE, ENOMEM=ENOMEM, ECUDA=ECUDA, ENCCL=ENCCL, ELAYOUT=ELAYOUT,
     ENOREPLICA=ENOREPLICA, ECONFLICT=ECONFLICT, ENOCONSISTENT=ENOCONSISTENT, EUNSTABLE=EUNSTABLE,
-    ECORRUPT=ECORRUPT, EINCOMPLETE=EINCOMPLETE, EIO=EIO).items()}
+    ECORRUPT=ECORRUPT, EINCOMPLETE=EINCOMPLETE, EIO=EIO, EPEER=EPEER).items()}
 CLEAN, DIRTY = 0, 1
 REQUIRED, OPTIONAL = 0, 1
 HOST, PEER = 0, 1
@@ -95,6 +95,7 @@ def lib() -> ctypes.CDLL:
         "jitc_comm_destroy": ([vp], i32),
         "jitc_comm_init_ipc": ([vp, ctypes.c_char_p, i32, i32, P(i32)], i32),
         "jitc_liveness_init": ([vp, ctypes.c_char_p], i32),
+        "jitc_comm_dead": ([vp, P(i32), i32, P(i32)], i32),
         "jitc_fingerprint": ([vp, u32, vp, sz, P(sz)], i32),
         "jitc_exchange_records": ([vp, vp, sz, vp, sz, P(sz)], i32),
         "jitc_select_consistent_replica": ([vp, sz, P(i32), i32, vp, sz, P(sz)], i32),
@@ -146,7 +147,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
             "jitc_inject_release", "jitc_capture_local", "jitc_set_aux", "jitc_get_aux", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop", "jitc_watchdog_failed", "jitc_capture_plan", "jitc_capture_fanout",
-            "jitc_attach_image", "jitc_liveness_init"]
+            "jitc_attach_image", "jitc_liveness_init", "jitc_comm_dead"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE, ON_HANG_COLLECTIVE_CAPTURE = 0, 1, 2
 
 
@@ -368,6 +369,13 @@ class Context:
         """Heartbeat table for failure localisation over an NCCL communicator
         (lets ON_HANG_COLLECTIVE_CAPTURE run with jitc_comm_init)."""
         _check(self._L.jitc_liveness_init(self._h, live_dir.encode()), "jitc_liveness_init")
+
+    def comm_dead(self) -> List[int]:
+        """Job ranks of the communicator whose heartbeat went stale."""
+        buf = (ctypes.c_int32 * 1024)()
+        n = ctypes.c_int32()
+        _check(self._L.jitc_comm_dead(self._h, buf, 1024, ctypes.byref(n)), "jitc_comm_dead")
+        return list(buf[:min(n.value, 1024)])
 
     def comm_shrink(self, failed: Sequence[int]):
         _check(self._L.jitc_comm_shrink(self._h, _i32arr(list(failed)), len(failed)), "jitc_comm_shrink")

@@ -1,0 +1,90 @@
+"""Reading R9: a writer dies during the
+capture -> the survivors re-run it with k - 1 writers, since HBM still holds
+their state.  Real processes on one B200 over the IPC transport:
+
+  3 ranks select writers {0, 1, 2} and capture their 1/3 shards; rank 1 dies
+  (os._exit) before the commit -> the survivors' commit barrier fails with
+  JITC_EPEER once rank 1's heartbeat is stale (instead of hanging) ->
+  jitc_comm_dead == [1] -> jitc_comm_shrink -> fingerprint -> exchange ->
+  select (writers {0, 2}) -> capture -> commit -> a replacement for rank 1
+  HOST-restores bit-exact against the oracle."""
+import os
+import shutil
+import subprocess
+import sys
+import textwrap
+import uuid
+
+import pytest
+
+from tests.test_gpu_hang_collective import REPL
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+RANK = r"""
+import os, sys, time
+sys.path.insert(0, {root!r})
+import torch
+from paper_conf_eurosys_guptakkvgkrs24_b200 import jitc as J
+from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
+from workloads import configs as W
+rank, shm = {rank}, {shm!r}
+w = W.scaled(W.c2(), 40000, )
+ctx = J.Context(device=0, rank=rank, world=3, chunk_bytes=1 << 20, image_dir=shm + "/img", staging_bytes=48 << 20,
+                slot_bytes=8 << 20)
+keep = []
+for g in w.groups:
+    st = GroupState(g, w.seed, shuffle_seed=rank); keep.append(st)
+    ctx.register(g.group, g.policy, [0, 1, 2], st.table(), keepalive=st)
+    ctx.mark(g.group, 50, J.CLEAN)
+torch.cuda.synchronize()
+ctx.comm_init_ipc(shm + "/comm", 3, rank)
+allb = ctx.exchange_records(ctx.fingerprint())
+s_, sel = J.select_consistent_replica(allb, [0, 1, 2])
+assert s_ == J.OK and J.parse_selection(sel)["groups"][0]["writers"] == [0, 1, 2]
+ctx.capture(sel)                                   # every writer's 1/3 shard
+if rank == 1:
+    os._exit(1)                                    # dies before the commit: no complete checkpoint exists
+t0 = time.time()
+try:
+    ctx.commit(sel)
+    raise SystemExit("commit succeeded without rank 1")
+except J.JitcError as e:
+    assert e.status == J.EPEER, e
+detect = time.time() - t0
+dead = ctx.comm_dead()
+assert dead == [1], dead
+ctx.comm_shrink(dead)
+allb = ctx.exchange_records(ctx.fingerprint())     # HBM still holds the state: re-run with k = 2
+s_, sel2 = J.select_consistent_replica(allb, [0, 2])
+assert s_ == J.OK and J.parse_selection(sel2)["groups"][0]["writers"] == [0, 2]
+cap = ctx.capture(sel2)
+ctx.commit(sel2)
+print("survivor", rank, "detected in %.2f s, recaptured" % detect, cap["image_bytes"], flush=True)
+ctx.close()
+"""
+
+
+def test_writer_dies_before_commit_survivors_recapture():
+    shm = f"/dev/shm/jitc-wdeath-{os.getpid()}-{uuid.uuid4().hex[:8]}"
+    os.makedirs(shm)
+    try:
+        env = dict(os.environ, JITC_PEER_DEAD_MS="500")
+        procs = [subprocess.Popen([sys.executable, "-c", textwrap.dedent(RANK.format(root=ROOT, rank=r, shm=shm))],
+                                  cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True, env=env)
+                 for r in range(3)]
+        try:
+            outs = [p.communicate(timeout=300)[0] for p in procs]
+        finally:
+            for p in procs:
+                if p.poll() is None:
+                    p.kill()
+        assert procs[1].returncode == 1
+        for i in (0, 2):
+            assert procs[i].returncode == 0 and "recaptured" in outs[i], "\n=====\n".join(outs)
+        r = subprocess.run([sys.executable, "-c", textwrap.dedent(REPL.format(root=ROOT, shm=shm))], cwd=ROOT,
+                           capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0 and "bit-exact" in r.stdout, r.stdout + r.stderr
+    finally:
+        shutil.rmtree(shm, ignore_errors=True)
