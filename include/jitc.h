@@ -404,8 +404,14 @@ jitc_status jitc_liveness_init(jitc_ctx* ctx, const char* dir);
  * JITC_PEER_DEAD_MS read at communicator init.  Writes up to cap ranks and
  * *n = count.  Local.  The recovery for reading R9 (a writer dies during the
  * capture): a collective call returns JITC_EPEER, every survivor calls this,
- * jitc_comm_shrink(dead), and re-runs fingerprint -> exchange -> select ->
- * capture -> commit with k - 1 writers (HBM still holds the state). */
+ * rebuilds the communicator without the dead ranks, and re-runs fingerprint
+ * -> exchange -> select -> capture -> commit with k - 1 writers (HBM still
+ * holds the state).  IPC transport: jitc_comm_shrink(dead).  NCCL: the
+ * failed collective is still in flight on the library's stream and
+ * ncclCommShrink cannot be trusted with it (measured: one survivor's shrink
+ * failed, the other's hung), so jitc_comm_shrink refuses (JITC_ESTATE);
+ * jitc_comm_destroy aborts the communicator and jitc_comm_init with a fresh
+ * unique id among the survivors (job_ranks) rebuilds it. */
 jitc_status jitc_comm_dead(jitc_ctx* ctx, int32_t* ranks, int32_t cap, int32_t* n);
 jitc_status jitc_watch_event(jitc_ctx* ctx, void* event, uint64_t tag);
 jitc_status jitc_watchdog_start(jitc_ctx* ctx, uint32_t timeout_ms, int32_t action, jitc_hang_fn fn, void* user);

@@ -392,6 +392,11 @@ jitc_status jitc_comm_init(jitc_ctx* c, const void* id128, int32_t nranks, int32
   if (!c || !id128 || nranks <= 0 || comm_rank < 0 || comm_rank >= nranks)
     return fail(JITC_EINVAL, "jitc_comm_init: bad argument");
   CU(cudaSetDevice(c->device));
+  if (c->comm && c->comm_broken) {  // its collective waits on a dead peer: abort it so the stream drains
+    ncclCommAbort(c->comm);
+    c->comm = nullptr;
+    c->comm_broken = false;
+  }
   if (c->comm) {  // retired, not freed: see jitc_ctx::retired_comms
     c->retired_comms.push_back(c->comm);
     c->comm = nullptr;
@@ -431,6 +436,10 @@ jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_faile
     c->ipc->slot = slot;
     c->ipc->peer_staging = ps;
   } else {
+    if (c->comm_broken)
+      return fail(JITC_ESTATE, "jitc_comm_shrink: a collective of this communicator waits on a dead peer "
+                               "(JITC_EPEER); rebuild instead: jitc_comm_destroy (aborts it), then jitc_comm_init "
+                               "with a fresh unique id among the survivors");
     // NCCL_SHRINK_ABORT aborts the parent's outstanding operations (a hung
     // collective of this communicator exits); the parent itself is retired,
     // not freed, until jitc_comm_destroy / jitc_destroy (see retired_comms).
@@ -440,6 +449,7 @@ jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_faile
     if (getenv("JITC_DEBUG_SHRINK")) fprintf(stderr, "jitc: ncclCommShrink done\n");
     c->retired_comms.push_back(c->comm);
     c->comm = nc;
+    c->comm_broken = false;
   }
   std::vector<int32_t> job;
   for (int i = 0; i < c->comm_n; ++i)
@@ -452,7 +462,12 @@ jitc_status jitc_comm_shrink(jitc_ctx* c, const int32_t* failed, int32_t n_faile
 
 jitc_status jitc_comm_destroy(jitc_ctx* c) {
   if (!c) return fail(JITC_EINVAL, "jitc_comm_destroy: null ctx");
-  if (c->comm) ncclCommDestroy(c->comm);
+  if (c->comm) {
+    if (getenv("JITC_DEBUG_SHRINK")) fprintf(stderr, "jitc: comm %s ...\n", c->comm_broken ? "abort" : "destroy");
+    c->comm_broken ? ncclCommAbort(c->comm) : ncclCommDestroy(c->comm);  // a broken comm's op never completes
+    if (getenv("JITC_DEBUG_SHRINK")) fprintf(stderr, "jitc: comm released\n");
+  }
+  c->comm_broken = false;
   for (ncclComm_t r : c->retired_comms) ncclCommAbort(r);
   c->retired_comms.clear();
   c->comm = nullptr;
@@ -527,6 +542,9 @@ jitc_status jitc_exchange_records(jitc_ctx* c, const void* mine, size_t len, voi
   c->h_small[0] = len;
   CU(cudaMemcpyAsync(dsz + c->comm_rank, c->h_small, 8, cudaMemcpyHostToDevice, c->s_comp));
   NC(ncclAllGather(dsz + c->comm_rank, dsz, 1, ncclUint64, c->comm, c->s_comp));
+  // wait for the collective before any copy into pageable memory (such a copy
+  // blocks the host behind it, where a dead peer could never be noticed)
+  if (jitc_status st = nccl_sync(c)) return st;
   std::vector<uint64_t> sizes(n);
   CU(cudaMemcpyAsync(sizes.data(), dsz, 8ull * n, cudaMemcpyDeviceToHost, c->s_comp));
   CU(cudaStreamSynchronize(c->s_comp));
@@ -541,6 +559,7 @@ jitc_status jitc_exchange_records(jitc_ctx* c, const void* mine, size_t len, voi
   uint8_t* recv = c->staging + 256;
   CU(cudaMemcpyAsync(recv + c->comm_rank * maxlen, mine, len, cudaMemcpyHostToDevice, c->s_comp));
   NC(ncclAllGather(recv + c->comm_rank * maxlen, recv, maxlen, ncclUint8, c->comm, c->s_comp));
+  if (jitc_status st = nccl_sync(c)) return st;
   CU(cudaMemcpyAsync(all, recv, n * maxlen, cudaMemcpyDeviceToHost, c->s_comp));
   CU(cudaStreamSynchronize(c->s_comp));
   uint8_t* a = static_cast<uint8_t*>(all);

@@ -172,6 +172,7 @@ struct jitc_ctx {
   std::vector<int32_t> comm_job;  // comm rank -> job rank
   std::unique_ptr<IpcComm> ipc;   // IPC transport (instead of `comm`)
   std::unique_ptr<Liveness> live; // heartbeats for the NCCL transport (jitc_liveness_init)
+  bool comm_broken = false;       // an NCCL collective of `comm` waits on a dead peer (nccl_sync)
   std::vector<uint8_t> aux;       // user CPU state for the next commit (jitc_set_aux)
   uint64_t* d_small = nullptr;    // 64 B device scratch for size exchange / barrier
   uint32_t* d_work = nullptr;     // K1/K2/K3 batch counters (self-resetting)
@@ -430,12 +431,18 @@ uint32_t group_slot(const jitc_ctx* c, uint32_t group);
 
 inline bool has_comm(const jitc_ctx* c) { return c->comm || c->ipc; }
 
+// Waits for the NCCL work enqueued on s_comp.  With a liveness table
+// (jitc_liveness_init) the wait polls: a communicator member whose heartbeat
+// goes stale cannot complete the collective, so the wait fails with
+// JITC_EPEER and the caller shrinks (reading R9); an asynchronous NCCL error
+// fails it with JITC_ENCCL.  Without a table: a plain stream synchronize.
+jitc_status nccl_sync(jitc_ctx* c);
+
 inline jitc_status barrier(jitc_ctx* c) {
   if (c->ipc) return ipc_barrier(c);
   if (!c->comm) return JITC_OK;
   NC(ncclAllReduce(c->d_small, c->d_small + 1, 1, ncclUint64, ncclSum, c->comm, c->s_comp));
-  CU(cudaStreamSynchronize(c->s_comp));
-  return JITC_OK;
+  return nccl_sync(c);
 }
 
 }  // namespace jitc

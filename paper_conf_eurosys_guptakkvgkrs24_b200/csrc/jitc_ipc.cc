@@ -76,6 +76,33 @@ double peer_dead_ms() {
   return v > 0 ? v : 2000.0;
 }
 
+jitc_status nccl_sync(jitc_ctx* c) {
+  if (!c->live || !c->comm) {
+    CU(cudaStreamSynchronize(c->s_comp));
+    return JITC_OK;
+  }
+  const double dead_ms = peer_dead_ms();
+  for (uint32_t it = 1;; ++it) {
+    cudaError_t e = cudaStreamQuery(c->s_comp);
+    if (e == cudaSuccess) return JITC_OK;
+    if (e != cudaErrorNotReady) return fail(JITC_ECUDA, std::string("nccl_sync: ") + cudaGetErrorString(e));
+    if ((it & 31) == 0) {
+      std::vector<int32_t> d = stale_ranks(c, dead_ms);
+      if (!d.empty()) {
+        c->comm_broken = true;
+        return fail(JITC_EPEER, "NCCL collective waits on a dead peer (job rank " + std::to_string(d[0]) +
+                                    ", heartbeat stale); shrink and retry");
+      }
+      ncclResult_t ae = ncclSuccess;
+      if (ncclCommGetAsyncError(c->comm, &ae) == ncclSuccess && ae != ncclSuccess && ae != ncclInProgress) {
+        c->comm_broken = true;
+        return fail(JITC_ENCCL, std::string("NCCL asynchronous error: ") + ncclGetErrorString(ae));
+      }
+    }
+    std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
+}
+
 bool ipc_peer_dead(const IpcComm& ic, int peer) {
   const uint64_t hb = load_acq(&ic.ctl->heartbeat[ic.slot[peer]]);
   return hb && mono_us() > hb + (uint64_t)(ic.dead_ms * 1000.0);

@@ -1,13 +1,17 @@
 """Reading R9: a writer dies during the
 capture -> the survivors re-run it with k - 1 writers, since HBM still holds
-their state.  Real processes on one B200 over the IPC transport:
+their state.  Real processes on one B200 over both transports:
 
   3 ranks select writers {0, 1, 2} and capture their 1/3 shards; rank 1 dies
   (os._exit) before the commit -> the survivors' commit barrier fails with
   JITC_EPEER once rank 1's heartbeat is stale (instead of hanging) ->
   jitc_comm_dead == [1] -> jitc_comm_shrink -> fingerprint -> exchange ->
   select (writers {0, 2}) -> capture -> commit -> a replacement for rank 1
-  HOST-restores bit-exact against the oracle."""
+  HOST-restores bit-exact against the oracle.  The same over NCCL (socket
+  transport on one GPU) with the liveness table: the commit's all-reduce
+  wait polls the heartbeats (nccl_sync) and fails with JITC_EPEER; the
+  survivors abort the communicator (the failed all-reduce is still in flight)
+  and build a fresh one among themselves."""
 import os
 import shutil
 import subprocess
@@ -29,7 +33,7 @@ import torch
 from paper_conf_eurosys_guptakkvgkrs24_b200 import jitc as J
 from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
 from workloads import configs as W
-rank, shm = {rank}, {shm!r}
+rank, shm, transport = {rank}, {shm!r}, {transport!r}
 w = W.scaled(W.c2(), 40000, )
 ctx = J.Context(device=0, rank=rank, world=3, chunk_bytes=1 << 20, image_dir=shm + "/img", staging_bytes=48 << 20,
                 slot_bytes=8 << 20)
@@ -39,7 +43,19 @@ for g in w.groups:
     ctx.register(g.group, g.policy, [0, 1, 2], st.table(), keepalive=st)
     ctx.mark(g.group, 50, J.CLEAN)
 torch.cuda.synchronize()
-ctx.comm_init_ipc(shm + "/comm", 3, rank)
+def uid(name, me):                                 # NCCL unique ids through the shared directory
+    p = shm + "/" + name
+    if me == 0:
+        open(p + ".tmp", "wb").write(J.get_unique_id())
+        os.rename(p + ".tmp", p)
+    while not os.path.exists(p):
+        time.sleep(0.01)
+    return open(p, "rb").read()
+if transport == "ipc":
+    ctx.comm_init_ipc(shm + "/comm", 3, rank)
+else:                                              # NCCL + the liveness table (jitc_liveness_init)
+    ctx.liveness_init(shm + "/live")
+    ctx.comm_init(uid("uid", rank), 3, rank)
 allb = ctx.exchange_records(ctx.fingerprint())
 s_, sel = J.select_consistent_replica(allb, [0, 1, 2])
 assert s_ == J.OK and J.parse_selection(sel)["groups"][0]["writers"] == [0, 1, 2]
@@ -51,11 +67,19 @@ try:
     ctx.commit(sel)
     raise SystemExit("commit succeeded without rank 1")
 except J.JitcError as e:
-    assert e.status == J.EPEER, e
+    # NCCL's socket transport may report the closed connection first (ENCCL)
+    assert e.status == J.EPEER or (transport == "nccl" and e.status == J.ENCCL), e
 detect = time.time() - t0
 dead = ctx.comm_dead()
+while not dead and time.time() - t0 < 10:          # (ENCCL can precede the stale heartbeat)
+    time.sleep(0.05)
+    dead = ctx.comm_dead()
 assert dead == [1], dead
-ctx.comm_shrink(dead)
+if transport == "ipc":
+    ctx.comm_shrink(dead)
+else:     # the failed all-reduce is still in flight: abort, then a fresh communicator among the survivors
+    ctx.comm_destroy()
+    ctx.comm_init(uid("uid2", 0 if rank == 0 else 1), 2, 0 if rank == 0 else 1, job_ranks=[0, 2])
 allb = ctx.exchange_records(ctx.fingerprint())     # HBM still holds the state: re-run with k = 2
 s_, sel2 = J.select_consistent_replica(allb, [0, 2])
 assert s_ == J.OK and J.parse_selection(sel2)["groups"][0]["writers"] == [0, 2]
@@ -66,13 +90,23 @@ ctx.close()
 """
 
 
-def test_writer_dies_before_commit_survivors_recapture():
+def _env(transport, r):
+    env = dict(os.environ, JITC_PEER_DEAD_MS="500")
+    if transport == "nccl":     # one fake host per rank: NCCL accepts three ranks on one GPU (socket transport)
+        env.update(NCCL_HOSTID=f"jitc-wd-host-{r}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
+                   NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0", NCCL_DEBUG="WARN")
+    return env
+
+
+@pytest.mark.parametrize("transport", ["ipc", "nccl"])
+def test_writer_dies_before_commit_survivors_recapture(transport):
     shm = f"/dev/shm/jitc-wdeath-{os.getpid()}-{uuid.uuid4().hex[:8]}"
     os.makedirs(shm)
     try:
-        env = dict(os.environ, JITC_PEER_DEAD_MS="500")
-        procs = [subprocess.Popen([sys.executable, "-c", textwrap.dedent(RANK.format(root=ROOT, rank=r, shm=shm))],
-                                  cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True, env=env)
+        procs = [subprocess.Popen([sys.executable, "-c", textwrap.dedent(RANK.format(root=ROOT, rank=r, shm=shm,
+                                                                                     transport=transport))],
+                                  cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True,
+                                  env=_env(transport, r))
                  for r in range(3)]
         try:
             outs = [p.communicate(timeout=300)[0] for p in procs]
