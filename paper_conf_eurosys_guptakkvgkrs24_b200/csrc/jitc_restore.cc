@@ -70,7 +70,7 @@ static jitc_status load_manifest(jitc_ctx* c, GroupState& g, ManifestView* mv) {
 jitc_status jitc::compare_digests(jitc_ctx* c, GroupState& g, const std::vector<uint64_t>& want, jitc_stats* stats) {
   if (g.n_c) {
     CU(cudaMemcpyAsync(c->h_dig, g.d_dig2, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
-    CU(cudaStreamSynchronize(c->s_comp));
+    if (jitc_status st = nccl_sync(c)) return st;  // NCCL rounds may wait on a dead peer
   }
   for (uint64_t ch = 0; ch < g.n_c; ++ch)
     if (c->h_dig[ch] != want[ch]) {
@@ -347,6 +347,7 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   }
   std::vector<uint64_t> want(g.n_c);
   if (is_dst) {
+    if (jitc_status st2 = nccl_sync(c)) return st2;  // the digest hand-off may wait on a dead writer
     if (g.n_c) CU(cudaMemcpyAsync(want.data(), d_expect, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
     CU(cudaStreamSynchronize(c->s_comp));
     if (root_of(g.layout_hash, want.data(), g.n_c) != gs.root)
@@ -360,7 +361,8 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   if (is_writer) readers = in.dests;
   st = execute_plan(c, g, ops, S, J, readers, stats);
   if (st) return st;
-  CU(cudaStreamSynchronize(c->s_comp));
+  st = nccl_sync(c);
+  if (st) return st;
   if (is_dst) {
     st = compare_digests(c, g, want, stats);
     if (st) return st;

@@ -122,3 +122,48 @@ def test_writer_dies_before_commit_survivors_recapture(transport):
         assert r.returncode == 0 and "bit-exact" in r.stdout, r.stdout + r.stderr
     finally:
         shutil.rmtree(shm, ignore_errors=True)
+
+
+PEER_RANK = RANK.split("ctx.capture(sel)")[0].replace(
+    'assert s_ == J.OK and J.parse_selection(sel)["groups"][0]["writers"] == [0, 1, 2]\n', "") + r"""
+# PEER restore: writers 0 and 1 rebuild rank 2 from live HBM; writer 1 dies first
+s_, sel = J.select_consistent_replica(allb, [0, 1])
+assert s_ == J.OK and J.parse_selection(sel)["groups"][0]["writers"] == [0, 1]
+if rank == 1:
+    os._exit(1)
+t0 = time.time()
+try:
+    ctx.restore(J.ALL_GROUPS, J.PEER, sel)
+    out = "completed"
+except J.JitcError as e:
+    assert e.status == J.EPEER or (transport == "nccl" and e.status == J.ENCCL), e
+    out = "EPEER" if e.status == J.EPEER else "ENCCL"
+print("rank", rank, out, "after %.2f s" % (time.time() - t0), flush=True)
+os._exit(0)                      # a failed survivor leaves (its heartbeat stops)
+"""
+
+
+@pytest.mark.parametrize("transport", ["ipc", "nccl"])
+def test_writer_dies_during_peer_restore_no_hang(transport):
+    """A writer dies before a PEER restore: the replacement's restore fails
+    with JITC_EPEER (NCCL's socket transport may report ENCCL first) within
+    seconds instead of hanging, and the other writer finishes or fails the
+    same way once the replacement has left."""
+    shm = f"/dev/shm/jitc-wdeathp-{os.getpid()}-{uuid.uuid4().hex[:8]}"
+    os.makedirs(shm)
+    try:
+        procs = [subprocess.Popen([sys.executable, "-c", textwrap.dedent(PEER_RANK.format(
+            root=ROOT, rank=r, shm=shm, transport=transport))], cwd=ROOT, stdout=subprocess.PIPE,
+            stderr=subprocess.STDOUT, text=True, env=_env(transport, r)) for r in range(3)]
+        try:
+            outs = [p.communicate(timeout=240)[0] for p in procs]
+        finally:
+            for p in procs:
+                if p.poll() is None:
+                    p.kill()
+        assert procs[1].returncode == 1
+        assert procs[2].returncode == 0 and ("rank 2 EPEER" in outs[2] or "rank 2 ENCCL" in outs[2]), \
+            "\n=====\n".join(outs)
+        assert procs[0].returncode == 0 and "rank 0 " in outs[0], "\n=====\n".join(outs)
+    finally:
+        shutil.rmtree(shm, ignore_errors=True)
