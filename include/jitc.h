@@ -111,8 +111,9 @@ typedef struct {
     uint64_t staging_bytes;  /* staging size; 0 => 1 GiB.  Split into rounds of slot_bytes.  */
     uint64_t slot_bytes;     /* bytes per pipeline round (multiple of C); 0 => 256 MiB       */
     const char* image_dir;   /* host image location: a directory on /dev/shm shared by the
-                                ranks of one box (survives process death), or NULL =>
-                                private pinned memory (writers must stay alive)               */
+                                ranks of one box (survives process death; the library never
+                                deletes it -- the launcher removes it when the job ends), or
+                                NULL => private pinned memory (writers must stay alive)       */
     void* streams[2];        /* caller-created non-blocking cudaStream_t (compute, copy) or
                                 NULL => library-created                                       */
 } jitc_config;
