@@ -19,6 +19,7 @@ from __future__ import annotations
 
 import argparse
 import json
+import numpy as np
 import os
 import shutil
 import statistics
@@ -206,31 +207,6 @@ def host_link_roofline(L_total, world, capture_ms, restore_ms, links):
 
 
 # ---------------------------------------------------------------------- reference arm / cpu baseline
-def oracle_sample(cfg_name: str, sample_bytes: int):
-    """Generates a bounded, contiguous prefix of the configuration's REQUIRED
-    group (same generator, same layout) on the host; not timed."""
-    import numpy as np
-    from oracle import oracle as O
-    from workloads import configs as W
-    w = W.CONFIGS[cfg_name]()
-    g = w.groups[0]
-    tensors, total = [], 0
-    import copy
-    g2 = copy.deepcopy(g)
-    g2.tensors = []
-    for t in g.tensors:
-        if total >= sample_bytes:
-            break
-        t2 = copy.deepcopy(t)
-        eb = W.ELEM_BYTES[t.dtype]
-        t2.numel = min(t.numel, max(1, (sample_bytes - total) // eb))
-        g2.tensors.append(t2)
-        total += t2.nbytes
-    lay = O.layout_of_group(g2, 1 << 20)
-    ts = O.gen_group(g2, w.seed)
-    return g2, lay, ts, total
-
-
 def cpu_model() -> str:
     try:
         for line in open("/proc/cpuinfo"):
@@ -248,65 +224,153 @@ def host_threads() -> int:
         return os.cpu_count() or 1
 
 
-def oracle_step(lay, ts, threads: int = 1):
-    """The oracle's capture+restore of the sample: pack + JF64 (capture),
-    JF64 verify + unpack (restore).  Plain C, as it stands; threads > 1 runs
-    the same calls on disjoint tensor runs / chunk ranges."""
-    import numpy as np
-    from oracle import oracle as O
-    img = O.pack(ts, lay, threads=threads)
-    d = O.jf64(img, lay.C, 0, lay.n_c, threads=threads)
-    d2 = O.jf64(img, lay.C, 0, lay.n_c, threads=threads)
-    assert np.array_equal(d, d2)
-    out = O.unpack(img, lay, threads=threads)
-    return out
+class OracleRecover:
+    """The oracle's capture + restore of one replica,
+    phase by phase: layout (O1), pack (O2), JF64 (O3: the fingerprint), select
+    (O6), shard (O5), unpack + verify (O3 over the image, compare with the
+    digests, O8).  State generation (O9) is not timed.  Pack and unpack+verify
+    run on every `every`-th chunk of each group (evenly spaced, chunk_sample)
+    and are extrapolated to the whole image by bytes; JF64 runs over the whole
+    committed /dev/shm image when one is given (the bytes the GPU digested, so
+    it doubles as a bit-exact check of the K1 digests), else on the sample.
+    Every step calls the oracle as it stands; `threads` runs the same calls on
+    disjoint chunk / tensor ranges."""
+
+    def __init__(self, w, rank: int, every: int, C: int = 1 << 20):
+        from oracle import oracle as O
+        from oracle import stream as S
+        self.O, self.S, self.w, self.every, self.C = O, S, w, every, C
+        self.groups = w.groups_of(rank)
+        self.lays = {g.group: O.layout_of_group(g, C) for g in self.groups}
+        self.samples = {g.group: S.chunk_sample(g, w.seed, self.lays[g.group], every) for g in self.groups}
+        self.L = sum(l.L for l in self.lays.values())
+        self.sample_bytes = sum(cs.nbytes for cs in self.samples.values())
+
+    def run(self, threads: int, blob: bytes = None, committed: dict = None, digests: dict = None) -> dict:
+        """One recovery of the replica; returns per-phase seconds (sampled
+        phases extrapolated), the measured (unextrapolated) seconds, and the
+        digest checks.  blob: this rank's record blob for O6 (built from the
+        sample's own digests when None); committed: group -> image array;
+        digests: group -> the GPU's K1 digests to check against."""
+        O, S = self.O, self.S
+        ph, meas, checks = {}, {}, {}
+        t = time.perf_counter()
+        lays = {g.group: O.layout_of_group(g, self.C) for g in self.groups}
+        ph["layout"] = meas["layout"] = time.perf_counter() - t
+        imgs, scale = {}, {}
+        t = time.perf_counter()
+        for gid, cs in self.samples.items():
+            imgs[gid] = O.pack(cs.pieces, cs.lay, threads=threads)
+        meas["pack"] = time.perf_counter() - t
+        ph["pack"] = meas["pack"] * self.L / max(self.sample_bytes, 1)
+        d_fp = {}
+        t = time.perf_counter()
+        if committed:
+            for gid, lay in lays.items():
+                d_fp[gid] = S.jf64_image(committed[gid], self.C, lay.L, threads)
+            meas["jf64"] = ph["jf64"] = time.perf_counter() - t
+            cover = "full"
+        else:
+            for gid, cs in self.samples.items():
+                d_fp[gid] = S.jf64_sample(imgs[gid], cs, lays[gid].n_c, threads)
+            meas["jf64"] = time.perf_counter() - t
+            ph["jf64"] = meas["jf64"] * self.L / max(self.sample_bytes, 1)
+            cover = "sampled"
+        if digests:
+            for gid, d in d_fp.items():
+                idx = slice(None) if committed else self.samples[gid].chunks
+                bad = int(np.count_nonzero(np.asarray(d)[idx] != np.asarray(digests[gid])[idx]))
+                checks[gid] = {"chunks": int(np.asarray(d)[idx].size), "mismatch": bad, "coverage": cover}
+        if blob is None:
+            recs = [O.Record(0, g.group, g.policy, O.CLEAN, 1, lays[g.group].layout_hash, self.C, lays[g.group].L,
+                             d_fp[g.group], O.root(lays[g.group].layout_hash, d_fp[g.group])) for g in self.groups]
+            blob = O.encode_blob(0, [O.TopoEntry(g.group, g.policy, [0]) for g in self.groups], recs)
+        t = time.perf_counter()
+        sel = O.select(blob, [0])
+        ph["select"] = meas["select"] = time.perf_counter() - t
+        assert sel.status == O.OK, sel.status
+        t = time.perf_counter()
+        for gs in sel.groups:
+            for s_ in range(len(gs.writers)):
+                O.shard_bytes(gs.n_c, len(gs.writers), s_, gs.C, gs.L)
+        ph["shard"] = meas["shard"] = time.perf_counter() - t
+        t = time.perf_counter()
+        for gid, cs in self.samples.items():
+            d = S.jf64_sample(imgs[gid], cs, lays[gid].n_c, threads)
+            if not np.array_equal(d[cs.chunks], np.asarray(d_fp[gid])[cs.chunks]):
+                raise RuntimeError(f"oracle restore: group {gid} digests differ (ECORRUPT)")
+            O.unpack(imgs[gid], cs.lay, threads=threads)
+        meas["unpack_verify"] = time.perf_counter() - t
+        ph["unpack_verify"] = meas["unpack_verify"] * self.L / max(self.sample_bytes, 1)
+        total = sum(ph.values())
+        return {"phases_s": {k: round(v, 4) for k, v in ph.items()},
+                "measured_s": {k: round(v, 4) for k, v in meas.items()},
+                "s_to_recover": round(total, 3), "GBps": round(self.L / total / 1e9, 4),
+                "measured_total_s": round(sum(meas.values()), 3), "checks": checks}
 
 
-def cpu_baseline(cfg_name: str, sample_bytes: int = 2 << 30, reps: int = 8):
-    """The oracle on the box's host cores (all of them), plus its 1-thread
-    figure; bounded sample."""
-    g2, lay, ts, total = oracle_sample(cfg_name, sample_bytes)
+def cpu_baseline(w, rank: int, blob: bytes, committed: dict, digests: dict, every: int, every_1t: int) -> dict:
+    """SURVEY.md §8(d) d.7 on rank 0 at N = 1: the oracle's recovery of the
+    same replica on all host cores and on 1 core.  JF64 covers the whole
+    committed image at nproc threads (and checks every K1 digest); pack and
+    unpack+verify are sampled (1/every of the chunks, evenly spaced) and
+    extrapolated; the 1-core leg samples everything at 1/every_1t."""
     nth = host_threads()
-    out = {}
-    oracle_step(lay, ts, nth)                      # untimed warm-up
-    for th, r in ((nth, reps), (1, 1)):
-        t0 = time.perf_counter()
-        for _ in range(r):
-            oracle_step(lay, ts, th)
-        out[th] = (time.perf_counter() - t0) / r
-    dt = out[nth]
-    return {"value": round(lay.L / dt / 1e9, 4), "unit": "GB/s", "cores": nth, "kind": "oracle",
-            "sample": f"first {lay.L / 2**30:.2f} GiB of the {cfg_name} REQUIRED-group image "
-                      f"({len(lay.names)} tensors), pack+JF64+JF64+unpack, {reps} reps, {nth} threads",
-            "seconds_per_sample": round(dt, 3), "cpu_model": cpu_model(), "nproc": os.cpu_count(),
-            "single_thread": {"value": round(lay.L / out[1] / 1e9, 4), "cores": 1,
-                              "seconds_per_sample": round(out[1], 3)}}
+    rec = OracleRecover(w, rank, every)
+    t0 = time.perf_counter()
+    full = rec.run(nth, blob=blob, committed=committed, digests=digests)
+    del rec
+    rec1 = OracleRecover(w, rank, every_1t)
+    one = rec1.run(1, blob=blob, digests=digests)
+    wall = time.perf_counter() - t0
+    return {"value": full["GBps"], "unit": "GB/s", "cores": nth, "kind": "oracle",
+            "sample": f"{w.name}: whole replica ({rec1.L / 1e9:.2f} GB); JF64 over the committed /dev/shm image "
+                      f"(every chunk, checked against the K1 digests); pack and unpack+verify on 1/{every} of the "
+                      f"chunks, evenly spaced, extrapolated by bytes; {nth} threads",
+            "s_to_recover": full["s_to_recover"], "phases_s": full["phases_s"], "measured_s": full["measured_s"],
+            "coverage": {"layout": "full", "pack": f"sampled 1/{every}", "jf64": "full (committed image)",
+                         "select": "full", "shard": "full", "unpack_verify": f"sampled 1/{every}"},
+            "digest_check": full["checks"],
+            "single_thread": {"value": one["GBps"], "cores": 1, "s_to_recover": one["s_to_recover"],
+                              "phases_s": one["phases_s"],
+                              "sample": f"every phase sampled at 1/{every_1t} of the chunks, extrapolated"},
+            "cpu_model": cpu_model(), "nproc": os.cpu_count(), "wall_s": round(wall, 1)}
 
 
 def run_reference(args):
+    """The reference arm: the oracle as it stands, on the box's host cores, on
+    the same config, metric and unit (capture + restore GB/s of one replica).
+    Each step is the oracle's whole recovery path (OracleRecover.run) over an
+    evenly spaced 1/ref_every chunk sample of the replica -- bounded so that
+    --steps K --warmup W end within minutes; value = sampled bytes / step."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     from workloads import configs as W
-    g2, lay, ts, total = oracle_sample(args.config, args.ref_sample << 20)
+    w = W.CONFIGS[args.config](world=max(args.gpus, 2) if args.config == "C1" else args.gpus)
+    rec = OracleRecover(w, 0, args.ref_every)
     nth = host_threads()
     for _ in range(args.warmup):
-        oracle_step(lay, ts, nth)
+        rec.run(nth)
     t0 = time.perf_counter()
+    last = None
     for _ in range(args.steps):
-        oracle_step(lay, ts, nth)
+        last = rec.run(nth)
     dt = (time.perf_counter() - t0) / args.steps
-    v = lay.L / dt / 1e9
+    v = rec.sample_bytes / dt / 1e9
     line = {"impl": "reference", "metric": "JIT capture+restore GB/s", "value": round(v, 4), "unit": "GB/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic (O9 counter-based generator)",
-            "config": {"workload": W.CONFIGS[args.config]().name, "sample_bytes": lay.L,
-                       "note": "bounded prefix of the same workload's REQUIRED image; oracle pack+JF64+JF64+unpack"},
+            "config": {"workload": w.name, "image_bytes": rec.L, "sample_bytes": rec.sample_bytes,
+                       "note": f"oracle layout/pack/JF64/select/shard/unpack+verify over 1/{args.ref_every} of the "
+                               "chunks of every group, evenly spaced"},
             "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": nth, "kind": "oracle",
                              "cpu_model": cpu_model(),
-                             "sample": f"first {lay.L / 2**20:.0f} MiB of the {args.config} REQUIRED-group image, "
-                                       f"{nth} threads"},
+                             "sample": f"1/{args.ref_every} of the chunks of {w.name} ({rec.sample_bytes / 1e9:.2f} GB "
+                                       f"of {rec.L / 1e9:.1f} GB), evenly spaced, {nth} threads",
+                             "phases_s_last_step": last["measured_s"],
+                             "s_to_recover_extrapolated": last["s_to_recover"]},
             "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -376,10 +440,13 @@ def run_jitc(args):
     per = {"fingerprint": [], "select": [], "capture": [], "commit": [], "restore": [], "verify": []}
     launches = [0]
 
+    last_blob = [None]
+
     def step(record: bool):
         t = {}
         t0 = time.perf_counter()
         blob = ctx.fingerprint()
+        last_blob[0] = blob
         t1 = time.perf_counter()
         allb = ctx.exchange_records(blob)
         st_, sel = J.select_consistent_replica(allb, healthy)
@@ -585,7 +652,10 @@ def run_jitc(args):
         value = L_total / (ms_step * 1e-3) / 1e9
         e2e = L_total / (ms_step_wall * 1e-3) / 1e9
         med = {k: round(statistics.median(v), 3) for k, v in per.items()}
-        cap_ms, res_ms = med["capture"] + med["commit"], med["restore"]
+        # T_capture runs from jitc_fingerprint start to
+        # jitc_commit return; T_restore from jitc_restore start to jitc_verify OK
+        cap_ms = med["fingerprint"] + med["select"] + med["capture"] + med["commit"]
+        res_ms = med["restore"] + med["verify"]
         line = {
             "metric": "JIT capture+restore GB/s", "value": round(value, 3), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
@@ -600,9 +670,12 @@ def run_jitc(args):
                        "l2": f"state {L_total / 1e9:.1f} GB >> 126 MB L2; no flush needed", "setup_s": round(setup_s, 1)},
             "seconds_to_recover": round(ms_step * 1e-3, 4),
             "phases_ms_median": med,
-            "capture_GBps": round(L_total / world / (cap_ms * 1e-3) / 1e9, 3),
+            "capture_GBps": round(L_total / (cap_ms * 1e-3) / 1e9, 3),
             "restore_GBps": round(L_total / (res_ms * 1e-3) / 1e9, 3),
-            "host_link_roofline": host_link_roofline(L_total, world, med["capture"], res_ms, links),
+            "capture_restore_spans": {"T_capture_ms": round(cap_ms, 3), "T_restore_ms": round(res_ms, 3),
+                                      "how": "SURVEY.md d.6: T_capture = fingerprint + exchange/select + capture + "
+                                             "commit; T_restore = restore + verify (medians over the timed steps)"},
+            "host_link_roofline": host_link_roofline(L_total, world, med["capture"], med["restore"], links),
             "per_tensor_d2h_baseline": f3,
             "roofline": {"kernel": kinds[dom], "bound": "hbm", "achieved": round(achieved, 1) if achieved else None,
                          "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
@@ -628,8 +701,13 @@ def run_jitc(args):
             "watchdog_on_hang": on_hang,
             "clocks": clk.summary(),
         }
-        if not args.no_cpu_baseline:
-            line["cpu_baseline"] = cpu_baseline(args.config)
+        if not args.no_cpu_baseline and world == 1:
+            from oracle import oracle as O
+            [(_, _, _, recs)] = O.decode_blobs(last_blob[0])
+            committed = {gid: np.memmap(f"{shm}/g{gid}.img", dtype=np.uint8, mode="r") for gid in states}
+            line["cpu_baseline"] = cpu_baseline(w, rank, last_blob[0], committed, {r.group: r.d for r in recs},
+                                                args.cpu_every, args.cpu_every_1t)
+            del committed
         print(json.dumps(line), flush=True)
     ctx.close()
     if world > 1:
@@ -645,12 +723,14 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3"])
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3"],
+                    help="workload (SURVEY.md §8(d) d.1); C3 = Llama-3-8B, the north-star shape and the largest "
+                         "single-GPU config")
     ap.add_argument("--impl", default="jitc", choices=["jitc", "reference"])
-    ap.add_argument("--staging", type=int, default=8192, help="MiB of device staging")
-    ap.add_argument("--slot", type=int, default=4096,
-                    help="MiB per pipeline round (4 GiB: the ~45 us per-launch cost of running next to a copy-engine "
-                         "transfer is amortised over 8.6 GB of K2/K3 traffic; profiles/r01_slot_size.txt)")
+    ap.add_argument("--staging", type=int, default=16384, help="MiB of device staging (2 round slots)")
+    ap.add_argument("--slot", type=int, default=8192,
+                    help="MiB per pipeline round (8 GiB: the ~42 us cost of a timing-event record next to a "
+                         "copy-engine transfer is amortised over 17 GB of K2/K3 traffic; DESIGN.md §7)")
     ap.add_argument("--zero-copy", action="store_true")
     ap.add_argument("--image-dir", default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -664,7 +744,11 @@ def main():
     ap.add_argument("--hang-ctas", type=int, default=32, help="CTAs of the emulated hung collective (0 = skip)")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nccl"],
                     help="N > 1 communicator: intra-node CUDA IPC (default; tested on B200 with real processes) or NCCL")
-    ap.add_argument("--ref-sample", type=int, default=1024, help="MiB per reference step")
+    ap.add_argument("--ref-every", type=int, default=128,
+                    help="reference arm: every step runs the oracle on 1/ref-every of the chunks")
+    ap.add_argument("--cpu-every", type=int, default=16,
+                    help="cpu_baseline: pack / unpack+verify sampled on 1/cpu-every of the chunks (1 = full state)")
+    ap.add_argument("--cpu-every-1t", type=int, default=128, help="cpu_baseline 1-thread leg: sample 1/N of the chunks")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

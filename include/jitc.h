@@ -98,7 +98,8 @@ enum {
     JITC_F_ZERO_COPY_D2H = 1u << 0,  /* capture: K2 stores straight into mapped pinned host memory */
     JITC_F_ZERO_COPY_H2D = 1u << 1,  /* restore: K3 loads straight from mapped pinned host memory  */
     JITC_F_TIME_KERNELS = 1u << 2,   /* bracket every kernel launch with CUDA events (stats)        */
-    JITC_F_NO_SHM_UNLINK = 1u << 3   /* keep /dev/shm images after a verified restore               */
+    JITC_F_RESERVED_3 = 1u << 3      /* reserved, no effect: the library never deletes host images
+                                        (image_dir belongs to the launcher)            */
 };
 
 typedef struct {
@@ -137,6 +138,10 @@ typedef struct {
     uint64_t kernel_launches;  /* launches of this library's kernels during the call           */
     uint32_t rounds;           /* pipeline rounds                                              */
     int32_t first_bad_chunk;   /* ECORRUPT: first chunk whose digest mismatched, else -1       */
+    uint32_t groups_done;      /* restore: groups restored by this call                         */
+    uint32_t groups_skipped;   /* restore: OPTIONAL groups left out -- dropped by the selection,
+                                  or (HOST without a selection) committed at a version other
+                                  than the REQUIRED groups' v* (reading R1)                    */
 } jitc_stats;
 
 /* Cumulative per-kernel counters (bench roofline): kind 1 = K1 digest,

@@ -9,6 +9,10 @@ using namespace jitc;
 // ------------------------------------------------------------ capture (K2 + D2H)
 static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelection& gs, uint64_t v_star,
                                  jitc_stats* stats) {
+  if (gs.writers.empty()) {  // dropped OPTIONAL group: no checkpoint of it may survive
+    drop_commit(c, g);
+    return JITC_OK;
+  }
   auto it = std::find(gs.writers.begin(), gs.writers.end(), c->cfg.rank);
   if (it == gs.writers.end()) return JITC_OK;  // not a writer
   uint64_t s = (uint64_t)(it - gs.writers.begin()), k = gs.writers.size();
@@ -48,7 +52,7 @@ static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelectio
         if (st) return st;
         CU(cudaEventRecord(c->ev_ready[sl], c->s_comp));
         CU(cudaStreamWaitEvent(c->s_copy, c->ev_ready[sl], 0));
-        CU(copy_pieces(c, g.img_h + a, slot, b - a, cudaMemcpyDeviceToHost, c->s_copy));
+        CU(copy_image(c, g, a, slot, b - a, cudaMemcpyDeviceToHost, c->s_copy));
         CU(cudaEventRecord(c->ev_free[sl], c->s_copy));
       }
       if (stats) stats->rounds += j;
@@ -215,7 +219,7 @@ static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection
       for (size_t q = i; q < e; ++q) {
         const PlanOp& op = ops[q];
         if (op.kind != kOpD2H) continue;
-        CU(copy_pieces(c, g.img_h + op.a, c->staging + op.off, op.bytes, cudaMemcpyDeviceToHost, c->s_copy));
+        CU(copy_image(c, g, op.a, c->staging + op.off, op.bytes, cudaMemcpyDeviceToHost, c->s_copy));
         if (stats) stats->d2h_bytes += op.bytes;
       }
       CU(cudaEventRecord(c->ev_free[sl], c->s_copy));
@@ -264,9 +268,12 @@ jitc_status jitc_capture_fanout(jitc_ctx* c, const void* selection, size_t sel_l
   CU(cudaEventRecord(c->ev_t0, c->s_comp));
   for (const GroupSelection& gs : sel.groups) {  // increasing group id on every rank
     if (group != JITC_ALL_GROUPS && gs.group != group) continue;
-    if (gs.writers.empty()) continue;  // dropped OPTIONAL group
     auto it = c->groups.find(gs.group);
     if (it == c->groups.end()) return fail(JITC_ELAYOUT, "jitc_capture_fanout: group unknown to this rank");
+    if (gs.writers.empty()) {  // dropped OPTIONAL group
+      if (it->second.held) drop_commit(c, it->second);
+      continue;
+    }
     jitc_status st = fanout_group(c, it->second, gs, sel.v_star, movers, n_movers, gen, stats);
     if (st) {
       harvest(c);
@@ -328,21 +335,19 @@ static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelec
   return b;
 }
 
-jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len, bool collective) {
-  if (!c) return fail(JITC_EINVAL, "jitc_commit: null ctx");
-  Selection sel;
-  std::string why;
-  if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
-    return fail(JITC_EINVAL, "jitc_commit: " + why);
-  if (sel.status != JITC_OK) return fail(sel.status, "jitc_commit: selection status is not OK");
-  CU(cudaSetDevice(c->device));
-  jitc_status st = collective ? barrier(c) : JITC_OK;  // every writer's capture has returned
-  if (st) return st;
+// The local part of jitc_commit: manifest + commit record of every group this
+// rank is the lowest writer of; dropped groups lose any older checkpoint.
+static jitc_status commit_groups(jitc_ctx* c, const Selection& sel) {
   for (auto& kv : c->groups) {
     GroupState& g = kv.second;
     if (!g.held) continue;
     const GroupSelection* gs = sel.find(g.id);
-    if (!gs || gs->writers.empty()) continue;
+    if (!gs) continue;
+    if (gs->writers.empty()) {
+      drop_commit(c, g);
+      g.has_man = false;
+      continue;
+    }
     bool writer = std::find(gs->writers.begin(), gs->writers.end(), c->cfg.rank) != gs->writers.end();
     if (!writer) continue;
     if (!g.captured || g.cap_v != sel.v_star) return fail(JITC_ESTATE, "jitc_commit: group not captured at v*");
@@ -366,7 +371,24 @@ jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len
         return fail(JITC_EIO, "jitc_commit: writing commit record: " + std::string(strerror(errno)));
     }
   }
-  return collective ? barrier(c) : JITC_OK;  // nobody restores before every commit record exists
+  return JITC_OK;
+}
+
+jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len, bool collective) {
+  if (!c) return fail(JITC_EINVAL, "jitc_commit: null ctx");
+  Selection sel;
+  std::string why;
+  if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
+    return fail(JITC_EINVAL, "jitc_commit: " + why);
+  if (sel.status != JITC_OK) return fail(sel.status, "jitc_commit: selection status is not OK");
+  CU(cudaSetDevice(c->device));
+  jitc_status st = collective ? barrier(c) : JITC_OK;  // every writer's capture has returned
+  if (st) return st;
+  st = commit_groups(c, sel);
+  // nobody restores before every commit record exists, and a rank that failed
+  // here (ESTATE, EIO) makes every rank fail with it instead of leaving them in
+  // a collective it never joins
+  return collective && has_comm(c) ? agree(c, st) : st;
 }
 
 jitc_status jitc_commit(jitc_ctx* c, const void* selection, size_t sel_len) {

@@ -15,10 +15,15 @@
 using namespace jitc;
 
 // ------------------------------------------------------------ fingerprint (K1)
+// The phase word is read twice, before K1 and after it completed (a seqlock):
+// a word that changed in between means the optimizer step that the hooks
+// bracket ran -- or started -- while K1 read the tensors, so the
+// digests may mix bytes from before and after it.  Such a record is labelled
+// DIRTY at the newer version and is never selected (reading R6); otherwise a
+// lone replica, guarded by its phase word alone (reading R12), could be
+// committed as CLEAN over torn bytes when the step stalls after K1.
 jitc_status jitc::fingerprint_group(jitc_ctx* c, GroupState& g) {
-  uint64_t w = __atomic_load_n(&c->phase_h[g.slot], __ATOMIC_ACQUIRE);
-  g.fp_version = w >> 1;
-  g.fp_phase = (int)(w & 1);
+  const uint64_t w = __atomic_load_n(&c->phase_h[g.slot], __ATOMIC_ACQUIRE);
   if (g.n_c) {
     CU(cudaMemsetAsync(g.d_dig, 0, g.n_c * 8, c->s_comp));
     jitc_status st = run_segments(c, g, kDigest, one_range(0, (uint32_t)g.segs.size(), nullptr, 0), g.d_dig, g.L);
@@ -26,10 +31,55 @@ jitc_status jitc::fingerprint_group(jitc_ctx* c, GroupState& g) {
     CU(cudaMemcpyAsync(c->h_dig, g.d_dig, g.n_c * 8, cudaMemcpyDeviceToHost, c->s_comp));
   }
   CU(cudaStreamSynchronize(c->s_comp));
+  if (c->debug_fp_pause_us) usleep(c->debug_fp_pause_us);
+  const uint64_t w2 = __atomic_load_n(&c->phase_h[g.slot], __ATOMIC_ACQUIRE);
+  g.fp_version = w2 >> 1;
+  g.fp_phase = (w2 != w) ? JITC_PHASE_DIRTY : (int)(w & 1);
   g.fp.assign(c->h_dig, c->h_dig + g.n_c);
   g.fp_root = root_of(g.layout_hash, g.fp.data(), g.n_c);
   g.has_fp = true;
+  g.captured = false;  // a capture belongs to the fingerprint it was checked against
   return JITC_OK;
+}
+
+// NCCL all-gather of one byte string per comm rank: the sizes first, then the
+// strings padded to the largest, in place in staging.
+static jitc_status nccl_gather(jitc_ctx* c, const void* mine, size_t len, std::vector<std::vector<uint8_t>>* parts) {
+  const int n = c->comm_n;
+  uint64_t* dsz = reinterpret_cast<uint64_t*>(c->staging);
+  c->h_small[0] = len;
+  CU(cudaMemcpyAsync(dsz + c->comm_rank, c->h_small, 8, cudaMemcpyHostToDevice, c->s_comp));
+  NC(ncclAllGather(dsz + c->comm_rank, dsz, 1, ncclUint64, c->comm, c->s_comp));
+  // wait for the collective before any copy into pageable memory (such a copy
+  // blocks the host behind it, where a dead peer could never be noticed)
+  if (jitc_status st = nccl_sync(c)) return st;
+  std::vector<uint64_t> sizes(n);
+  CU(cudaMemcpyAsync(sizes.data(), dsz, 8ull * n, cudaMemcpyDeviceToHost, c->s_comp));
+  CU(cudaStreamSynchronize(c->s_comp));
+  uint64_t maxlen = 0;
+  for (uint64_t s : sizes) maxlen = std::max(maxlen, s);
+  maxlen = align_up(std::max<uint64_t>(maxlen, 1), 256);
+  if (256 + n * maxlen > c->staging_bytes) return fail(JITC_ENOMEM, "gather: blobs exceed staging");
+  uint8_t* recv = c->staging + 256;
+  if (len) CU(cudaMemcpyAsync(recv + c->comm_rank * maxlen, mine, len, cudaMemcpyHostToDevice, c->s_comp));
+  NC(ncclAllGather(recv + c->comm_rank * maxlen, recv, maxlen, ncclUint8, c->comm, c->s_comp));
+  if (jitc_status st = nccl_sync(c)) return st;
+  std::vector<uint8_t> all(n * maxlen);
+  CU(cudaMemcpyAsync(all.data(), recv, n * maxlen, cudaMemcpyDeviceToHost, c->s_comp));
+  CU(cudaStreamSynchronize(c->s_comp));
+  parts->assign(n, {});
+  for (int r = 0; r < n; ++r) (*parts)[r].assign(all.data() + r * maxlen, all.data() + r * maxlen + sizes[r]);
+  return JITC_OK;
+}
+
+jitc_status jitc::gather_bytes(jitc_ctx* c, const void* mine, size_t len, std::vector<std::vector<uint8_t>>* parts) {
+  if (c->ipc) return ipc_gather(c, mine, len, parts);
+  if (!c->comm) {
+    parts->assign(1, std::vector<uint8_t>(static_cast<const uint8_t*>(mine), static_cast<const uint8_t*>(mine) + len));
+    return JITC_OK;
+  }
+  CU(cudaSetDevice(c->device));
+  return nccl_gather(c, mine, len, parts);
 }
 
 // =====================================================================
@@ -112,6 +162,7 @@ jitc_status jitc_create(const jitc_config* cfg, jitc_ctx** out) {
     c->write_value64 = (PFN_writeValue64)fn;
   cudaGetLastError();
   c->grid = segment_grid(c->device);
+  if (const char* e = getenv("JITC_DEBUG_FP_PAUSE_US")) c->debug_fp_pause_us = (uint32_t)strtoul(e, nullptr, 10);
   *out = c.release();
   return JITC_OK;
 }
@@ -180,12 +231,26 @@ static jitc_status declare(jitc_ctx* c, uint32_t group, int32_t policy, const in
   return JITC_OK;
 }
 
+// Registration geometry of a shared image: pieces of kRegPiece bytes pinned
+// by up to kPinThreads threads at once.  One 32 GiB cudaHostRegister takes
+// 9.7 s on the pool's boxes; four concurrent 8 GiB ones take 3.9 s
+// (tools/pin_probe3.py, profiles/r02_pin_probe.txt).  JITC_PIN_THREADS
+// overrides the thread count (1 => one registration of the whole image).
+constexpr uint64_t kRegPiece = 1ull << 30;
+constexpr int kPinThreads = 4;
+
 // Maps image_dir/g<group>.img (g.img_bytes) shared and pins it (mapped,
 // portable).  Several ranks of a box register the same image.  Concurrent
-// cudaHostRegister calls that fault the same fresh tmpfs pages in fail
+// cudaHostRegister calls that fault the same FRESH tmpfs pages in fail
 // (error 304, measured with >= 8 GiB images: tools/pin_probe2.py), so the
-// pages are allocated up front (posix_fallocate, idempotent) and the
-// registration itself is serialised with an exclusive flock on the file.
+// file is sized and its pages allocated (posix_fallocate, idempotent) under
+// an exclusive flock first; the pages then exist and the registrations run
+// concurrently -- across the ranks of the box and, within a rank, over
+// 1 GiB pieces on several threads.  The pieces are adjacent in the device's
+// unified address space (the registered host address IS the device address
+// on this platform, cudaDevAttrCanUseHostPointerForRegisteredMem), so the
+// kernels see one contiguous mapping; copy_image keeps every copy-engine
+// transfer inside one piece.
 static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::string& who) {
   mkdir(c->image_dir.c_str(), 0700);
   g.img_path = gpath(c, g.id, ".img");
@@ -197,26 +262,47 @@ static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::strin
   if (fstat(fd, &sb) != 0 || ((uint64_t)sb.st_size != g.img_bytes && ftruncate(fd, (off_t)g.img_bytes) != 0))
     err = errno ? errno : EIO;
   if (!err) err = posix_fallocate(fd, 0, (off_t)g.img_bytes);
+  flock(fd, LOCK_UN);
   if (err) {
-    flock(fd, LOCK_UN);
     close(fd);
     return fail(JITC_EIO, who + ": sizing " + g.img_path + ": " + strerror(err));
   }
   void* p = mmap(nullptr, g.img_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
-  if (p == MAP_FAILED) {
-    flock(fd, LOCK_UN);
-    close(fd);
-    return fail(JITC_EIO, who + ": mmap " + g.img_path + ": " + strerror(errno));
-  }
-  cudaError_t e = cudaHostRegister(p, g.img_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
-  flock(fd, LOCK_UN);
   close(fd);
-  if (e != cudaSuccess) {
-    munmap(p, g.img_bytes);
-    return fail(JITC_ENOMEM, who + ": cudaHostRegister: " + cudaGetErrorString(e));
-  }
+  if (p == MAP_FAILED) return fail(JITC_EIO, who + ": mmap " + g.img_path + ": " + strerror(errno));
+  int same = 0;
+  cudaDeviceGetAttribute(&same, cudaDevAttrCanUseHostPointerForRegisteredMem, c->device);
+  int threads = kPinThreads;
+  if (const char* e = getenv("JITC_PIN_THREADS")) threads = std::max(1, atoi(e));
+  uint64_t reg_piece = kRegPiece;  // JITC_PIN_PIECE_MB: tests cross piece boundaries with small images
+  if (const char* e = getenv("JITC_PIN_PIECE_MB")) reg_piece = std::max<uint64_t>(1, strtoull(e, nullptr, 10)) << 20;
+  const uint64_t piece = (same && threads > 1 && g.img_bytes > reg_piece) ? reg_piece : g.img_bytes;
+  const uint64_t n_pieces = (g.img_bytes + piece - 1) / piece;
+  std::vector<cudaError_t> rc(n_pieces, cudaSuccess);
+  std::atomic<uint64_t> next{0};
+  auto work = [&] {
+    cudaSetDevice(c->device);
+    for (uint64_t i; (i = next++) < n_pieces;) {
+      const uint64_t a = i * piece, n = std::min(piece, g.img_bytes - a);
+      rc[i] = cudaHostRegister(static_cast<uint8_t*>(p) + a, n, cudaHostRegisterMapped | cudaHostRegisterPortable);
+    }
+  };
+  std::vector<std::thread> pool;
+  for (int t = 1; t < threads && (uint64_t)t < n_pieces; ++t) pool.emplace_back(work);
+  work();
+  for (auto& th : pool) th.join();
   g.img_h = (uint8_t*)p;
   g.img_shm = true;
+  g.img_reg_piece = n_pieces > 1 ? piece : 0;
+  cudaError_t bad = cudaSuccess;
+  for (uint64_t i = 0; i < n_pieces; ++i) {
+    if (rc[i] == cudaSuccess) g.img_regs.push_back(g.img_h + i * piece);
+    else if (bad == cudaSuccess) bad = rc[i];
+  }
+  if (bad != cudaSuccess) {
+    release_image(g);
+    return fail(JITC_ENOMEM, who + ": cudaHostRegister: " + cudaGetErrorString(bad));
+  }
   return JITC_OK;
 }
 
@@ -309,9 +395,7 @@ jitc_status jitc_attach_image(jitc_ctx* c, uint32_t group, uint64_t image_bytes)
   GroupState& g = it->second;
   if (g.img_h) {
     if (g.L == image_bytes) return JITC_OK;
-    cudaHostUnregister(g.img_h);
-    munmap(g.img_h, g.img_bytes);
-    g.img_h = g.img_d = nullptr;
+    release_image(g);
   }
   g.L = image_bytes;
   g.img_bytes = align_up(image_bytes, 4096);
@@ -535,40 +619,20 @@ jitc_status jitc_exchange_records(jitc_ctx* c, const void* mine, size_t len, voi
     memcpy(all, mine, len);
     return JITC_OK;
   }
-  CU(cudaSetDevice(c->device));
-  const int n = c->comm_n;
-  // 1. sizes
-  uint64_t* dsz = reinterpret_cast<uint64_t*>(c->staging);
-  c->h_small[0] = len;
-  CU(cudaMemcpyAsync(dsz + c->comm_rank, c->h_small, 8, cudaMemcpyHostToDevice, c->s_comp));
-  NC(ncclAllGather(dsz + c->comm_rank, dsz, 1, ncclUint64, c->comm, c->s_comp));
-  // wait for the collective before any copy into pageable memory (such a copy
-  // blocks the host behind it, where a dead peer could never be noticed)
-  if (jitc_status st = nccl_sync(c)) return st;
-  std::vector<uint64_t> sizes(n);
-  CU(cudaMemcpyAsync(sizes.data(), dsz, 8ull * n, cudaMemcpyDeviceToHost, c->s_comp));
-  CU(cudaStreamSynchronize(c->s_comp));
-  uint64_t maxlen = 0, total = 0;
-  for (uint64_t s : sizes) maxlen = std::max(maxlen, s), total += s;
-  maxlen = align_up(maxlen, 256);
-  *all_len = (size_t)(n * maxlen);   // capacity needed (the compacted result is `total` <= this)
+  // both calls of the size query run the whole (small: <= 1 MB per rank) gather
+  std::vector<std::vector<uint8_t>> parts;
+  jitc_status st = gather_bytes(c, mine, len, &parts);
+  if (st) return st;
+  size_t total = 0;
+  for (auto& b : parts) total += b.size();
+  *all_len = total;
   if (cap == 0) return JITC_OK;
-  if (cap < n * maxlen || !all) return fail(JITC_EINVAL, "jitc_exchange_records: buffer too small");
-  if (256 + n * maxlen > c->staging_bytes) return fail(JITC_ENOMEM, "jitc_exchange_records: blobs exceed staging");
-  // 2. padded blobs, in place
-  uint8_t* recv = c->staging + 256;
-  CU(cudaMemcpyAsync(recv + c->comm_rank * maxlen, mine, len, cudaMemcpyHostToDevice, c->s_comp));
-  NC(ncclAllGather(recv + c->comm_rank * maxlen, recv, maxlen, ncclUint8, c->comm, c->s_comp));
-  if (jitc_status st = nccl_sync(c)) return st;
-  CU(cudaMemcpyAsync(all, recv, n * maxlen, cudaMemcpyDeviceToHost, c->s_comp));
-  CU(cudaStreamSynchronize(c->s_comp));
+  if (cap < total || !all) return fail(JITC_EINVAL, "jitc_exchange_records: buffer too small");
   uint8_t* a = static_cast<uint8_t*>(all);
-  uint64_t pos = 0;
-  for (int r = 0; r < n; ++r) {
-    memmove(a + pos, a + r * maxlen, sizes[r]);
-    pos += sizes[r];
+  for (auto& b : parts) {
+    memcpy(a, b.data(), b.size());
+    a += b.size();
   }
-  *all_len = (size_t)total;
   return JITC_OK;
 }
 

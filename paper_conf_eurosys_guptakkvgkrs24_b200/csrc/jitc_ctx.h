@@ -69,6 +69,10 @@ struct GroupState {
   uint8_t* img_d = nullptr;  // device alias of the mapped host image
   size_t img_bytes = 0;
   bool img_shm = false;
+  // a shared image is pinned as separate registrations of img_reg_piece bytes
+  // each (0: one registration); a host<->device copy must not cross one
+  uint64_t img_reg_piece = 0;
+  std::vector<uint8_t*> img_regs;
   std::string img_path;
   std::vector<uint8_t> man_priv, commit_priv;  // private-memory manifest / commit
 };
@@ -98,6 +102,9 @@ struct IpcCtl {
   // capture fan-out rounds: (call generation << 24) | (round + 1)
   uint64_t cap_posted[kIpcMaxRanks][kIpcMaxGroups];
   uint64_t cap_consumed[kIpcMaxRanks][kIpcMaxGroups];
+  // status agreement (jitc::agree): (generation << 16) | -status, two slots by
+  // generation parity -- a rank can be at most one barrier generation ahead
+  uint64_t agree[2][kIpcMaxRanks];
 };
 struct IpcComm {
   std::string dir;
@@ -107,9 +114,13 @@ struct IpcComm {
   std::vector<int> slot;               // comm rank -> index into the IpcCtl arrays (stable across shrink)
   std::vector<uint8_t*> peer_staging;  // by comm rank (own entry = ctx staging)
   std::vector<void*> opened;
-  uint64_t barrier_gen = 0, exchange_gen = 0, cap_gen = 0;
-  std::map<uint32_t, uint64_t> rounds;      // cumulative restore rounds per group slot
-  std::map<uint32_t, uint64_t> digest_gen;  // PEER digest hand-offs per group slot
+  uint64_t barrier_gen = 0, exchange_gen = 0, cap_gen = 0, agree_gen = 0;
+  // restore calls per group slot.  Every participant of a group's restore
+  // advances it once per call, before anything can fail, so a call that
+  // aborts part-way (JITC_EPEER, a timeout) leaves every survivor on the same
+  // generation; the round counters of call `gen` are (gen << 24) | (round + 1),
+  // so stale counter values of an aborted call never satisfy a later wait.
+  std::map<uint32_t, uint64_t> restore_gen;
   std::thread hb_thread;                    // heartbeat writer (failure localisation, NEXT-1)
   std::atomic<bool> hb_run{false};
   double dead_ms = 2000.0;                  // a peer whose heartbeat is older is dead (JITC_PEER_DEAD_MS)
@@ -196,7 +207,11 @@ struct jitc_ctx {
   void* hang_user = nullptr;
   jitc_status action_status = JITC_OK;
   jitc_stats action_stats{};
-  std::vector<int32_t> fired_failed;  // job ranks the collective action found dead
+  std::vector<int32_t> fired_failed;  // job ranks the collective action found dead (guarded by wmu)
+  std::string action_error;           // jitc_last_error text of a failed action (guarded by wmu)
+  // test hook (JITC_DEBUG_FP_PAUSE_US, read at create): pause between the end
+  // of K1 and the second phase-word read of jitc_fingerprint (seqlock test)
+  uint32_t debug_fp_pause_us = 0;
   // counters
   jitc_kernel_counter kc[5]{};
   uint64_t launches_in_call = 0;
@@ -296,14 +311,24 @@ inline void finish_stats(jitc_ctx* c, const CallTimer& t, jitc_stats* st, bool d
   }
 }
 
-// A host<->device copy on `s`, issued in pieces of at most c->copy_piece bytes.
-inline cudaError_t copy_pieces(const jitc_ctx* c, void* dst, const void* src, uint64_t n, cudaMemcpyKind kind,
-                               cudaStream_t s) {
+// A copy between image bytes [img_off, img_off + n) of group g and device
+// memory `dev`, issued in pieces of at most c->copy_piece bytes that never
+// cross a registration boundary of the pinned image (cudaMemcpy refuses a
+// host range that spans two registrations).
+inline cudaError_t copy_image(const jitc_ctx* c, const GroupState& g, uint64_t img_off, void* dev, uint64_t n,
+                              cudaMemcpyKind kind, cudaStream_t s) {
   const uint64_t P = c->copy_piece ? c->copy_piece : n;
-  for (uint64_t o = 0; o < n; o += P) {
-    cudaError_t e = cudaMemcpyAsync(static_cast<uint8_t*>(dst) + o, static_cast<const uint8_t*>(src) + o,
-                                    std::min(P, n - o), kind, s);
+  const uint64_t R = g.img_reg_piece;
+  uint64_t o = 0;
+  while (o < n) {
+    uint64_t len = std::min(P, n - o);
+    if (R) len = std::min(len, R - (img_off + o) % R);
+    uint8_t* h = g.img_h + img_off + o;
+    uint8_t* d = static_cast<uint8_t*>(dev) + o;
+    cudaError_t e = kind == cudaMemcpyDeviceToHost ? cudaMemcpyAsync(h, d, len, kind, s)
+                                                   : cudaMemcpyAsync(d, h, len, kind, s);
     if (e != cudaSuccess) return e;
+    o += len;
   }
   return cudaSuccess;
 }
@@ -347,23 +372,30 @@ inline jitc_status ensure_h_dig(jitc_ctx* c, size_t n) {
   return JITC_OK;
 }
 
+// Unpins and unmaps a shared image, or frees a private one.
+inline void release_image(GroupState& g) {
+  if (g.img_h) {
+    if (g.img_shm) {
+      for (uint8_t* r : g.img_regs) cudaHostUnregister(r);
+      munmap(g.img_h, g.img_bytes);
+    } else {
+      cudaFreeHost(g.img_h);
+    }
+  }
+  g.img_regs.clear();
+  g.img_reg_piece = 0;
+  g.img_h = g.img_d = nullptr;
+}
+
 inline void free_group(GroupState& g) {
   if (g.d_segs) cudaFree(g.d_segs);
   if (g.d_dig) cudaFree(g.d_dig);
   if (g.d_dig2) cudaFree(g.d_dig2);
   if (g.d_remote) cudaFree(g.d_remote);
   g.d_remote = nullptr;
-  if (g.img_h) {
-    if (g.img_shm) {
-      cudaHostUnregister(g.img_h);
-      munmap(g.img_h, g.img_bytes);
-    } else {
-      cudaFreeHost(g.img_h);
-    }
-  }
+  release_image(g);
   g.d_segs = nullptr;
   g.d_dig = g.d_dig2 = nullptr;
-  g.img_h = g.img_d = nullptr;
 }
 
 inline std::string gpath(const jitc_ctx* c, uint32_t g, const char* ext) {
@@ -398,6 +430,21 @@ inline bool write_file_atomic(const std::string& path, const uint8_t* p, size_t 
   return ok && rename(tmp.c_str(), path.c_str()) == 0;
 }
 
+// A group the selection dropped (an OPTIONAL group with no candidate at v*,
+// reading R1) keeps no checkpoint: its commit record (and manifest) from an
+// earlier failure would otherwise stay valid at an older version and a later
+// HOST restore without a selection would load it.  Every member that holds the
+// group removes them (idempotent) at capture and again at commit.
+inline void drop_commit(jitc_ctx* c, GroupState& g) {
+  if (g.img_shm) {
+    unlink(gpath(c, g.id, ".commit").c_str());
+    unlink(gpath(c, g.id, ".manifest").c_str());
+  }
+  g.commit_priv.clear();
+  g.man_priv.clear();
+  g.captured = false;
+}
+
 inline bool read_file(const std::string& path, std::vector<uint8_t>* out) {
   FILE* f = fopen(path.c_str(), "rb");
   if (!f) return false;
@@ -415,6 +462,7 @@ namespace jitc {
 // IPC transport (jitc_ipc.cc)
 jitc_status ipc_barrier(jitc_ctx* c);
 jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len);
+jitc_status ipc_gather(jitc_ctx* c, const void* mine, size_t len, std::vector<std::vector<uint8_t>>* parts);
 jitc_status ipc_post(jitc_ctx* c, uint64_t* counter, uint64_t value, cudaStream_t s);
 jitc_status ipc_wait(const uint64_t* counter, uint64_t value, const char* what);
 // the same, failing with JITC_EPEER if comm rank `peer`'s heartbeat goes stale meanwhile
@@ -437,6 +485,16 @@ inline bool has_comm(const jitc_ctx* c) { return c->comm || c->ipc; }
 // JITC_EPEER and the caller shrinks (reading R9); an asynchronous NCCL error
 // fails it with JITC_ENCCL.  Without a table: a plain stream synchronize.
 jitc_status nccl_sync(jitc_ctx* c);
+
+// Every comm rank contributes its local status; all return the same one: the
+// first failing rank's code (lowest comm rank), JITC_OK if none failed.  A
+// collective call whose ranks can fail independently (jitc_commit) ends with
+// this instead of a plain barrier, so a failed rank neither leaves its peers
+// blocked in the next collective nor lets them report success.
+jitc_status agree(jitc_ctx* c, jitc_status mine);
+// All-gather of one byte string per comm rank (any length, 0 included), in
+// comm-rank order.  Collective; without a communicator returns {mine}.
+jitc_status gather_bytes(jitc_ctx* c, const void* mine, size_t len, std::vector<std::vector<uint8_t>>* parts);
 
 inline jitc_status barrier(jitc_ctx* c) {
   if (c->ipc) return ipc_barrier(c);

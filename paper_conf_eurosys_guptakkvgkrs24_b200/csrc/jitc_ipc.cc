@@ -146,25 +146,77 @@ jitc_status ipc_barrier(jitc_ctx* c) {
   return JITC_OK;
 }
 
-jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len) {
+// (failed ? (~comm_rank << 32) | -status : 0): the max over ranks is the
+// failing rank with the lowest comm rank, its status in the low word
+static uint64_t agree_word(const jitc_ctx* c, jitc_status st) {
+  return st ? ((uint64_t)(0xFFFFFFFFu - (uint32_t)c->comm_rank) << 32) | (uint32_t)(-st) : 0;
+}
+
+jitc_status agree(jitc_ctx* c, jitc_status mine) {
+  const std::string mine_err = mine ? get_error() : std::string();
+  uint64_t worst = agree_word(c, mine);
+  if (c->ipc) {
+    IpcComm& ic = *c->ipc;
+    const uint64_t gen = ++ic.agree_gen;
+    uint64_t* row = ic.ctl->agree[gen & 1];
+    // (generation << 40) | (failed ? 1 << 16 | -status : 0); the reader knows the rank
+    const uint64_t w = mine ? (1ull << 16) | (uint16_t)(-mine) : 0;
+    store_rel(&row[ic.slot[c->comm_rank]], (gen << 40) | w);
+    for (int q = 0; q < c->comm_n; ++q) {
+      const uint64_t* p = &row[ic.slot[q]];
+      jitc_status st = ipc_wait_peer(ic, q, p, gen << 40, "a status agreement");
+      if (st) return st;
+      const uint64_t v = load_acq(p) & ((1ull << 40) - 1);
+      if (v) {
+        const uint64_t full = ((0xFFFFFFFFull - (uint64_t)q) << 32) | (v & 0xFFFF);
+        worst = std::max(worst, full);
+      }
+    }
+  } else if (c->comm) {
+    c->h_small[2] = worst;
+    CU(cudaMemcpyAsync(c->d_small + 4, c->h_small + 2, 8, cudaMemcpyHostToDevice, c->s_comp));
+    NC(ncclAllReduce(c->d_small + 4, c->d_small + 5, 1, ncclUint64, ncclMax, c->comm, c->s_comp));
+    if (jitc_status st = nccl_sync(c)) return st;
+    CU(cudaMemcpyAsync(c->h_small + 3, c->d_small + 5, 8, cudaMemcpyDeviceToHost, c->s_comp));
+    CU(cudaStreamSynchronize(c->s_comp));
+    worst = c->h_small[3];
+  }
+  if (!worst) return JITC_OK;
+  const int who = (int)(0xFFFFFFFFu - (uint32_t)(worst >> 32));
+  const jitc_status code = -(jitc_status)(worst & 0xFFFF);
+  if (who == c->comm_rank) return fail(mine, mine_err);
+  if (mine) return fail(mine, mine_err);
+  return fail(code, "comm rank " + std::to_string(who) + " (job rank " +
+                        std::to_string(who >= 0 && who < (int)c->comm_job.size() ? c->comm_job[who] : -1) +
+                        ") failed with status " + std::to_string(code));
+}
+
+jitc_status ipc_gather(jitc_ctx* c, const void* mine, size_t len, std::vector<std::vector<uint8_t>>* parts) {
   IpcComm& ic = *c->ipc;
-  // the two-call size query is collective too: both calls run the protocol
+  // every gather (and each call of the two-call exchange size query) runs the
+  // whole protocol, so the generations stay in step on every rank
   const uint64_t gen = ++ic.exchange_gen;
   std::string me = ic.dir + "/blob." + std::to_string(gen) + "." + std::to_string(ic.slot[c->comm_rank]);
-  if (!write_file_atomic(me, static_cast<const uint8_t*>(mine), len))
-    return fail(JITC_EIO, "jitc_exchange_records: writing " + me);
+  if (!write_file_atomic(me, static_cast<const uint8_t*>(mine), len)) return fail(JITC_EIO, "IPC gather: writing " + me);
   jitc_status st = ipc_barrier(c);
   if (st) return st;
-  std::vector<uint8_t> out;
+  parts->assign(c->comm_n, {});
   for (int q = 0; q < c->comm_n; ++q) {
-    std::vector<uint8_t> b;
     std::string p = ic.dir + "/blob." + std::to_string(gen) + "." + std::to_string(ic.slot[q]);
-    if (!read_file(p, &b)) return fail(JITC_EIO, "jitc_exchange_records: reading " + p);
-    out.insert(out.end(), b.begin(), b.end());
+    if (!read_file(p, &(*parts)[q])) return fail(JITC_EIO, "IPC gather: reading " + p);
   }
   st = ipc_barrier(c);  // every rank has read every blob
   if (st) return st;
   unlink(me.c_str());
+  return JITC_OK;
+}
+
+jitc_status ipc_exchange(jitc_ctx* c, const void* mine, size_t len, void* all, size_t cap, size_t* all_len) {
+  std::vector<std::vector<uint8_t>> parts;
+  jitc_status st = ipc_gather(c, mine, len, &parts);
+  if (st) return st;
+  std::vector<uint8_t> out;
+  for (auto& b : parts) out.insert(out.end(), b.begin(), b.end());
   *all_len = out.size();
   if (cap == 0) return JITC_OK;
   if (cap < out.size() || !all) return fail(JITC_EINVAL, "jitc_exchange_records: buffer too small");

@@ -89,11 +89,12 @@ jitc_status jitc::compare_digests(jitc_ctx* c, GroupState& g, const std::vector<
 // and every rank posts / consumes every round (counters in shared memory)
 // so that senders know when a slot may be refilled.
 static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<PlanOp>& ops, uint32_t S, uint32_t J,
-                                const std::vector<int>& readers, jitc_stats* stats) {
+                                const std::vector<int>& readers, uint64_t gen, jitc_stats* stats) {
   if (S > (uint32_t)jitc_ctx::kSlots) return fail(JITC_EINVAL, "execute_plan: too many slots");
+  if (J >= (1u << 24)) return fail(JITC_EINVAL, "execute_plan: too many rounds");
   IpcComm* ic = c->ipc.get();
   const uint32_t gs = ic ? group_slot(c, g.id) : 0;
-  const uint64_t base_round = ic ? ic->rounds[gs] : 0;
+  const uint64_t base_round = gen << 24;  // IPC counters of this call: (gen << 24) | (round + 1)
   const int my_slot = ic ? ic->slot[c->comm_rank] : 0;
   bool used[jitc_ctx::kSlots] = {false};
   size_t i = 0;
@@ -120,7 +121,7 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
       if (op.kind != kOpH2D) continue;
       if (!any_h2d && used[sl]) CU(cudaStreamWaitEvent(c->s_copy, c->ev_free[sl], 0));
       any_h2d = true;
-      CU(copy_pieces(c, c->staging + op.off, g.img_h + op.a, op.bytes, cudaMemcpyHostToDevice, c->s_copy));
+      CU(copy_image(c, g, op.a, c->staging + op.off, op.bytes, cudaMemcpyHostToDevice, c->s_copy));
       if (stats) stats->h2d_bytes += op.bytes;
     }
     if (any_h2d) {
@@ -207,7 +208,6 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
       jitc_status st = ipc_wait_peer(*ic, r, &ic->ctl->consumed[ic->slot[r]][gs], base_round + J, "a peer to finish reading");
       if (st) return st;
     }
-    ic->rounds[gs] = base_round + J;
   }
   if (stats) stats->rounds += rounds;
   return JITC_OK;
@@ -223,10 +223,8 @@ static jitc_status make_plan(jitc_ctx* c, const PlanInput& in, std::vector<PlanO
 // HOST mode: this rank (or, with a communicator, every comm rank) loads a
 // 1/n slice of the committed image H2D; slices are all-gathered over NVLink
 // round by round and every round is unpacked+verified by K3.
-static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
-  ManifestView mv;
-  jitc_status st = load_manifest(c, g, &mv);
-  if (st) return st;
+static jitc_status restore_host(jitc_ctx* c, GroupState& g, const ManifestView& mv, uint64_t gen, jitc_stats* stats) {
+  jitc_status st = JITC_OK;
   if (g.n_c) CU(cudaMemsetAsync(g.d_dig2, 0, g.n_c * 8, c->s_comp));
   const int n = has_comm(c) ? c->comm_n : 1;
   if (n > 1 && !g.img_shm)
@@ -262,7 +260,7 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
     for (int r : in.participants)
       if (r != in.me) readers.push_back(r);
     if (std::find(in.participants.begin(), in.participants.end(), in.me) == in.participants.end()) readers.clear();
-    st = execute_plan(c, g, ops, S, J, readers, stats);
+    st = execute_plan(c, g, ops, S, J, readers, gen, stats);
     if (st) return st;
   }
   st = compare_digests(c, g, mv.d, stats);
@@ -278,7 +276,7 @@ static jitc_status restore_host(jitc_ctx* c, GroupState& g, jitc_stats* stats) {
 // PEER mode: the selection's writers pack their O5 ranges from live HBM (K2)
 // and send them over NVLink to every member that is not a writer; receivers
 // unpack+verify (K3) against the writers' digests (broadcast first).
-static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection& gs, jitc_stats* stats) {
+static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection& gs, uint64_t gen, jitc_stats* stats) {
   if (!has_comm(c)) return fail(JITC_ESTATE, "jitc_restore: PEER mode needs a communicator");
   if (gs.writers.empty()) return JITC_OK;  // dropped OPTIONAL group
   if (gs.layout_hash != g.layout_hash || gs.n_c != g.n_c || gs.image_bytes != g.L)
@@ -322,7 +320,6 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
     // IPC: the lowest writer leaves the digests in a file of the communicator
     // directory (per group and hand-off generation); receivers wait for it.
     const uint32_t gsl = group_slot(c, g.id);
-    const uint64_t gen = ++c->ipc->digest_gen[gsl];
     const std::string path = c->ipc->dir + "/dig." + std::to_string(gsl) + "." + std::to_string(gen);
     if (is_writer && my_s == 0 && !write_file_atomic(path, reinterpret_cast<const uint8_t*>(g.fp.data()), 8 * g.n_c))
       return fail(JITC_EIO, "jitc_restore: writing " + path);
@@ -359,7 +356,7 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   // 2. data rounds
   std::vector<int> readers;  // a writer's blocks are read by every destination
   if (is_writer) readers = in.dests;
-  st = execute_plan(c, g, ops, S, J, readers, stats);
+  st = execute_plan(c, g, ops, S, J, readers, gen, stats);
   if (st) return st;
   st = nccl_sync(c);
   if (st) return st;
@@ -381,33 +378,132 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   return JITC_OK;
 }
 
+// PEER mode without a selection on some ranks (a fresh replacement took no
+// part in the selection): every comm rank contributes the selection it holds
+// (or nothing) and all adopt the one of the lowest comm rank that has one --
+// the surviving writers computed it from the same all-gathered records, so
+// every selection present must be byte-identical (the
+// replacement gets the selection over the new communicator).  The writers'
+// digests follow in restore_peer's hand-off.
+static jitc_status share_selection(jitc_ctx* c, const void* selection, size_t sel_len, std::vector<uint8_t>* out) {
+  std::vector<std::vector<uint8_t>> parts;
+  jitc_status st = gather_bytes(c, selection, selection ? sel_len : 0, &parts);
+  if (st) return st;
+  out->clear();
+  for (auto& p : parts) {
+    if (p.empty()) continue;
+    if (out->empty()) {
+      *out = p;
+    } else if (p != *out) {
+      return fail(JITC_EINVAL, "jitc_restore: ranks passed different selections");
+    }
+  }
+  if (out->empty()) return fail(JITC_EINVAL, "jitc_restore: PEER mode needs the selection on at least one rank");
+  return JITC_OK;
+}
+
 jitc_status jitc_restore(jitc_ctx* c, uint32_t group, int32_t mode, const void* selection, size_t sel_len,
                          jitc_stats* stats) {
   NvtxRange nvtx_(mode == JITC_RESTORE_HOST ? "jitc_restore(HOST)" : "jitc_restore(PEER)");
   if (!c) return fail(JITC_EINVAL, "jitc_restore: null ctx");
   if (mode != JITC_RESTORE_HOST && mode != JITC_RESTORE_PEER) return fail(JITC_EINVAL, "jitc_restore: bad mode");
-  Selection sel;
-  bool have_sel = false;
-  if (selection) {
-    std::string why;
-    if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
-      return fail(JITC_EINVAL, "jitc_restore: " + why);
-    if (sel.status != JITC_OK) return fail(sel.status, "jitc_restore: selection status is not OK");
-    have_sel = true;
-  } else if (mode == JITC_RESTORE_PEER) {
-    return fail(JITC_EINVAL, "jitc_restore: PEER mode needs the selection");
-  }
   CU(cudaSetDevice(c->device));
   if (stats) memset(stats, 0, sizeof *stats), stats->first_bad_chunk = -1;
-  CallTimer t(c);
-  CU(cudaEventRecord(c->ev_t0, c->s_comp));
+  // the groups of this call; with the IPC transport each advances its restore
+  // generation first, so every participant stays on the same generation even
+  // if this call fails part-way on some rank
+  std::vector<GroupState*> todo;
+  std::map<uint32_t, uint64_t> gen;
   for (auto& kv : c->groups) {
     GroupState& g = kv.second;
     if (!g.held || (group != JITC_ALL_GROUPS && g.id != group)) continue;
-    const GroupSelection* gs = have_sel ? sel.find(g.id) : nullptr;
-    if (have_sel && !gs) return fail(JITC_ELAYOUT, "jitc_restore: group missing from selection");
-    if (gs && gs->writers.empty()) continue;  // dropped OPTIONAL group: nothing to restore
-    jitc_status st = mode == JITC_RESTORE_HOST ? restore_host(c, g, stats) : restore_peer(c, g, *gs, stats);
+    todo.push_back(&g);
+    gen[g.id] = c->ipc ? ++c->ipc->restore_gen[group_slot(c, g.id)] : 0;
+  }
+  // 1. the selection (PEER: shared from the ranks that have it)
+  Selection sel;
+  bool have_sel = false;
+  std::vector<uint8_t> shared;
+  jitc_status st = JITC_OK;
+  if (mode == JITC_RESTORE_PEER && has_comm(c)) {
+    st = share_selection(c, selection, sel_len, &shared);
+    if (!st) selection = shared.data(), sel_len = shared.size();
+  } else if (mode == JITC_RESTORE_PEER && !selection) {
+    st = fail(JITC_EINVAL, "jitc_restore: PEER mode needs the selection");
+  }
+  if (!st && selection) {
+    std::string why;
+    if (!parse_selection(static_cast<const uint8_t*>(selection), sel_len, &sel, &why))
+      st = fail(JITC_EINVAL, "jitc_restore: " + why);
+    else if (sel.status != JITC_OK)
+      st = fail(sel.status, "jitc_restore: selection status is not OK");
+    have_sel = !st;
+  }
+  // 2. what each group restores from.  HOST: its committed manifest, whose v*
+  //    must be the selection's, or -- without a selection -- the one v* of the
+  //    REQUIRED groups; an OPTIONAL group committed at another version is
+  //    stale (its checkpoint predates a failure that dropped it) and is left
+  //    out, as a dropped group is (reading R1).  PEER: the selection's entry.
+  std::map<uint32_t, ManifestView> man;
+  std::vector<GroupState*> run;
+  uint32_t skipped = 0;
+  if (!st) {
+    for (GroupState* g : todo) {
+      const GroupSelection* gs = have_sel ? sel.find(g->id) : nullptr;
+      if (have_sel && !gs) {
+        st = fail(JITC_ELAYOUT, "jitc_restore: group " + std::to_string(g->id) + " missing from selection");
+        break;
+      }
+      if (gs && gs->writers.empty()) {  // dropped OPTIONAL group: nothing to restore
+        ++skipped;
+        continue;
+      }
+      if (mode == JITC_RESTORE_HOST) {
+        st = load_manifest(c, *g, &man[g->id]);
+        if (st == JITC_EINCOMPLETE && !have_sel && g->policy == JITC_OPTIONAL) {
+          st = JITC_OK;  // no checkpoint of this OPTIONAL group: the last selection dropped it
+          ++skipped;
+          continue;
+        }
+        if (st) break;
+        if (have_sel && man[g->id].h.v_star != sel.v_star) {
+          st = fail(JITC_EINCOMPLETE, "jitc_restore: group " + std::to_string(g->id) + " is committed at version " +
+                                          std::to_string(man[g->id].h.v_star) + ", the selection's v* is " +
+                                          std::to_string(sel.v_star));
+          break;
+        }
+      } else if (gs->layout_hash != g->layout_hash || gs->n_c != g->n_c || gs->image_bytes != g->L) {
+        st = fail(JITC_ELAYOUT, "jitc_restore: selection layout differs from the registered one");
+        break;
+      }
+      run.push_back(g);
+    }
+  }
+  if (!st && mode == JITC_RESTORE_HOST && !have_sel) {
+    std::vector<uint64_t> req;
+    for (GroupState* g : run)
+      if (g->policy == JITC_REQUIRED) req.push_back(man[g->id].h.v_star);
+    std::sort(req.begin(), req.end());
+    req.erase(std::unique(req.begin(), req.end()), req.end());
+    if (req.size() > 1) {
+      st = fail(JITC_EINCOMPLETE, "jitc_restore: REQUIRED groups are committed at different versions (" +
+                                      std::to_string(req.front()) + " .. " + std::to_string(req.back()) + ")");
+    } else if (req.size() == 1) {
+      std::vector<GroupState*> keep;
+      for (GroupState* g : run)
+        if (g->policy == JITC_REQUIRED || man[g->id].h.v_star == req[0]) keep.push_back(g);
+        else ++skipped;
+      run.swap(keep);
+    }
+  }
+  // every rank fails together before any data moves (restore is collective)
+  if (has_comm(c)) st = agree(c, st);
+  if (st) return st;
+  CallTimer t(c);
+  CU(cudaEventRecord(c->ev_t0, c->s_comp));
+  for (GroupState* g : run) {
+    st = mode == JITC_RESTORE_HOST ? restore_host(c, *g, man[g->id], gen[g->id], stats)
+                                   : restore_peer(c, *g, *sel.find(g->id), gen[g->id], stats);
     if (st) {
       harvest(c);
       return st;
@@ -416,6 +512,7 @@ jitc_status jitc_restore(jitc_ctx* c, uint32_t group, int32_t mode, const void* 
   CU(cudaEventRecord(c->ev_t1, c->s_comp));
   CU(cudaEventSynchronize(c->ev_t1));
   finish_stats(c, t, stats, true);
+  if (stats) stats->groups_done = (uint32_t)run.size(), stats->groups_skipped = skipped;
   return JITC_OK;
 }
 

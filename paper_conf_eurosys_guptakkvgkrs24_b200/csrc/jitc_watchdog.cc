@@ -29,7 +29,10 @@ static jitc_status collective_capture(jitc_ctx* c, jitc_stats* st) {
     r = jitc_comm_shrink(c, failed.data(), (int32_t)failed.size());
     if (r) return r;
   }
-  c->fired_failed = failed;
+  {
+    std::lock_guard<std::mutex> lk(c->wmu);  // read by jitc_watchdog_failed on other threads
+    c->fired_failed = failed;
+  }
   size_t len = 0;
   r = jitc_fingerprint(c, JITC_ALL_GROUPS, nullptr, 0, &len);
   if (r) return r;
@@ -85,9 +88,12 @@ static void watchdog_loop(jitc_ctx* c) {
       if (c->action == JITC_ON_HANG_LOCAL_CAPTURE || c->action == JITC_ON_HANG_COLLECTIVE_CAPTURE) {
         jitc_stats st{};
         jitc_status r = c->action == JITC_ON_HANG_LOCAL_CAPTURE ? local_capture(c, &st) : collective_capture(c, &st);
+        // the error text is thread-local: hand this thread's to jitc_watchdog_wait
+        const std::string err = r ? get_error() : std::string();
         lk.lock();
         c->action_status = r;
         c->action_stats = st;
+        c->action_error = err;
         lk.unlock();
       }
       if (c->hang_fn) c->hang_fn(c->hang_user, c->fired_tag, c->waited_ms);
@@ -132,6 +138,8 @@ jitc_status jitc_watchdog_start(jitc_ctx* c, uint32_t timeout_ms, int32_t action
   c->hang_user = user;
   c->fired = c->action_done = false;
   c->action_status = JITC_OK;
+  c->action_error.clear();
+  c->fired_failed.clear();
   c->action_stats = jitc_stats{};
   c->action_stats.first_bad_chunk = -1;
   c->wrun = true;
@@ -150,7 +158,8 @@ jitc_status jitc_watchdog_wait(jitc_ctx* c, uint32_t max_ms, int32_t* fired, uin
   if (action_ms) *action_ms = c->action_ms;
   if (action_stats) *action_stats = c->action_stats;
   jitc_status st = c->action_done ? c->action_status : JITC_OK;
-  if (st) set_error("jitc_watchdog_wait: the on-hang capture failed with status " + std::to_string(st));
+  if (st) set_error("jitc_watchdog_wait: the on-hang capture failed with status " + std::to_string(st) + ": " +
+                    c->action_error);
   return st;
 }
 

@@ -27,8 +27,11 @@ STATUS_NAMES = {v: k for k, v in dict(
 CLEAN, DIRTY = 0, 1
 REQUIRED, OPTIONAL = 0, 1
 HOST, PEER = 0, 1
+# per-group selection status (jitc_sel_group.status) and exclusion reasons (include/jitc.h)
+G_OK, G_UNVERIFIED_SINGLE, G_NOREPLICA, G_DROPPED, G_CONFLICT, G_NOCANDIDATE = 0, 1, 2, 3, 4, 5
+X_DIRTY, X_STALE_VERSION, X_MINORITY = 1, 2, 3
 ALL_GROUPS = 0xFFFFFFFF
-F_ZERO_COPY_D2H, F_ZERO_COPY_H2D, F_TIME_KERNELS, F_NO_SHM_UNLINK = 1, 2, 4, 8
+F_ZERO_COPY_D2H, F_ZERO_COPY_H2D, F_TIME_KERNELS = 1, 2, 4   # bit 3 is reserved (no effect)
 K_DIGEST, K_PACK, K_UNPACK, K_PULL = 1, 2, 3, 4
 
 
@@ -55,7 +58,8 @@ class Stats(ctypes.Structure):
     _fields_ = [("ms_host", ctypes.c_double), ("ms_device", ctypes.c_double), ("ms_kernel", ctypes.c_double),
                 ("image_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64), ("h2d_bytes", ctypes.c_uint64),
                 ("p2p_bytes", ctypes.c_uint64), ("kernel_launches", ctypes.c_uint64), ("rounds", ctypes.c_uint32),
-                ("first_bad_chunk", ctypes.c_int32)]
+                ("first_bad_chunk", ctypes.c_int32), ("groups_done", ctypes.c_uint32),
+                ("groups_skipped", ctypes.c_uint32)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
