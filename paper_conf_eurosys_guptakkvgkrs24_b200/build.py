@@ -53,22 +53,26 @@ def _run(cmd):
     subprocess.check_call(cmd)
 
 
-def build(force: bool = False, verbose_ptxas: bool = False, sanitize: bool = False) -> str:
+def build(force: bool = False, verbose_ptxas: bool = False, sanitize: bool = False, tsan: bool = False) -> str:
     """sanitize=True builds libjitc_asan.so: host code with AddressSanitizer +
-    UndefinedBehaviorSanitizer (tests/test_asan.py drives it; not the product)."""
+    UndefinedBehaviorSanitizer (tests/test_asan.py drives it); tsan=True builds
+    libjitc_tsan.so: host code with ThreadSanitizer (tests/test_tsan.py).
+    Neither is the product."""
     cuda, nccl = _cuda_home(), _nccl_home()
     nvcc = os.path.join(cuda, "bin", "nvcc")
     nccl_lib = os.path.join(nccl, "lib") if os.path.isdir(os.path.join(nccl, "lib")) else "/usr/lib/x86_64-linux-gnu"
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cc")))
     hdrs = sorted(glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(INCLUDE, "*.h")))
-    out = OUT.replace("libjitc.so", "libjitc_asan.so") if sanitize else OUT
-    bdir = BUILD + ("_asan" if sanitize else "")
+    out = OUT.replace("libjitc.so", "libjitc_asan.so") if sanitize else \
+        OUT.replace("libjitc.so", "libjitc_tsan.so") if tsan else OUT
+    bdir = BUILD + ("_asan" if sanitize else "_tsan" if tsan else "")
     newest = max(os.path.getmtime(p) for p in srcs + hdrs + [__file__])
     if not force and os.path.exists(out) and os.path.getmtime(out) >= newest:
         return out
     os.makedirs(bdir, exist_ok=True)
     san = ["-Xcompiler", "-fsanitize=address", "-Xcompiler", "-fsanitize=undefined", "-Xcompiler",
-           "-fno-omit-frame-pointer", "-Xcompiler", "-g"] if sanitize else []
+           "-fno-omit-frame-pointer", "-Xcompiler", "-g"] if sanitize else \
+        ["-Xcompiler", "-fsanitize=thread", "-Xcompiler", "-fno-omit-frame-pointer", "-Xcompiler", "-g"] if tsan else []
     incs = ["-I", INCLUDE, "-I", CSRC, "-I", os.path.join(nccl, "include")]
     objs = []
     for s in srcs:
@@ -90,4 +94,5 @@ def build(force: bool = False, verbose_ptxas: bool = False, sanitize: bool = Fal
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose_ptxas="-v" in sys.argv, sanitize="--asan" in sys.argv)
+    build(force="--force" in sys.argv, verbose_ptxas="-v" in sys.argv, sanitize="--asan" in sys.argv,
+          tsan="--tsan" in sys.argv)

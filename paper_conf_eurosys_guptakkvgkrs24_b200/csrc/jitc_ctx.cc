@@ -254,6 +254,7 @@ constexpr int kPinThreads = 4;
 static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::string& who) {
   mkdir(c->image_dir.c_str(), 0700);
   g.img_path = gpath(c, g.id, ".img");
+  const double t_open = now_ms();
   int fd = open(g.img_path.c_str(), O_RDWR | O_CREAT, 0600);
   if (fd < 0) return fail(JITC_EIO, who + ": open " + g.img_path + ": " + strerror(errno));
   flock(fd, LOCK_EX);
@@ -267,6 +268,7 @@ static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::strin
     close(fd);
     return fail(JITC_EIO, who + ": sizing " + g.img_path + ": " + strerror(err));
   }
+  const double t_sized = now_ms();
   void* p = mmap(nullptr, g.img_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
   close(fd);
   if (p == MAP_FAILED) return fail(JITC_EIO, who + ": mmap " + g.img_path + ": " + strerror(errno));
@@ -291,6 +293,10 @@ static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::strin
   for (int t = 1; t < threads && (uint64_t)t < n_pieces; ++t) pool.emplace_back(work);
   work();
   for (auto& th : pool) th.join();
+  if (getenv("JITC_DEBUG_TIMING"))
+    fprintf(stderr, "jitc: %s group %u: %.2f GB sized in %.0f ms, pinned in %.0f ms (%llu pieces, %d threads)\n",
+            who.c_str(), g.id, g.img_bytes / 1e9, t_sized - t_open, now_ms() - t_sized,
+            (unsigned long long)n_pieces, threads);
   g.img_h = (uint8_t*)p;
   g.img_shm = true;
   g.img_reg_piece = n_pieces > 1 ? piece : 0;

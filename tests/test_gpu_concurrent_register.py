@@ -20,8 +20,10 @@ import sys, time
 sys.path.insert(0, {root!r})
 import torch
 from paper_conf_eurosys_guptakkvgkrs24_b200 import jitc as J
+device = {rank} % torch.cuda.device_count()
+torch.cuda.set_device(device)
 x = torch.empty(12 << 30, dtype=torch.uint8, device="cuda")
-ctx = J.Context(device=0, rank={rank}, world=3, image_dir={shm!r}, staging_bytes=64 << 20, slot_bytes=16 << 20)
+ctx = J.Context(device=device, rank={rank}, world=3, image_dir={shm!r}, staging_bytes=64 << 20, slot_bytes=16 << 20)
 while time.time() < {start}:
     time.sleep(0.001)
 t = time.time()

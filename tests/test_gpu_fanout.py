@@ -38,6 +38,8 @@ from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
 from workloads import configs as W
 
 rank, shm, transport = {rank}, {shm!r}, {transport!r}
+device = rank % torch.cuda.device_count()
+torch.cuda.set_device(device)
 base = W.scaled(W.c2(), 40000).groups[0]
 groups = []
 for p in (0, 1):
@@ -49,12 +51,12 @@ seed = 0x4A4954435F563105
 
 RANK = SETUP + r"""
 comm = [0, 1, 2]
-ctx = J.Context(device=0, rank=rank, world=4, chunk_bytes={C}, image_dir=shm + "/img",
+ctx = J.Context(device=device, rank=rank, world=4, chunk_bytes={C}, image_dir=shm + "/img",
                 staging_bytes=24 << 20, slot_bytes=4 << 20, flags=J.F_TIME_KERNELS)
 st = None
 for g in groups:
     if rank in g.members:
-        st = GroupState(g, seed, shuffle_seed=3 + rank)
+        st = GroupState(g, seed, device=device, shuffle_seed=3 + rank)
         ctx.register(g.group, g.policy, g.members, st.table(), keepalive=st)
         ctx.mark(g.group, 12, J.CLEAN)
     else:
@@ -86,10 +88,10 @@ ctx.close()
 """
 
 REPLACEMENT = SETUP + r"""
-ctx = J.Context(device=0, rank=3, world=4, chunk_bytes={C}, image_dir=shm + "/img",
+ctx = J.Context(device=device, rank=3, world=4, chunk_bytes={C}, image_dir=shm + "/img",
                 staging_bytes=24 << 20, slot_bytes=4 << 20)
 g = groups[1]
-st = GroupState(g, seed, fill=False, shuffle_seed=11)
+st = GroupState(g, seed, device=device, fill=False, shuffle_seed=11)
 st.scramble()
 ctx.register(g.group, g.policy, g.members, st.table(), keepalive=st)
 ctx.declare_group(0, groups[0].policy, groups[0].members)
@@ -104,10 +106,8 @@ ctx.close()
 
 
 def _env(transport, rank):
-    if transport == "ipc":
-        return dict(os.environ)
-    return dict(os.environ, NCCL_HOSTID=f"jitc-fanout-host-{rank}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
-                NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0", NCCL_DEBUG="WARN")
+    from tests.mp_util import nccl_env
+    return dict(os.environ) if transport == "ipc" else nccl_env("fanout", rank)
 
 
 def _run(code, env):

@@ -39,14 +39,34 @@ groups.append(sub)
 seed = base.seed
 
 
-def make_ctx(comm_dir, scramble):
-    ctx = J.Context(device=0, rank=rank, world=world, chunk_bytes=1 << 20, image_dir=shm + "/img",
+# one process per GPU when the box has several (NVLink / NVSwitch: NCCL P2P and
+# NVLS, CUDA IPC peer loads); all on GPU 0 of a 1-GPU box
+device = rank % torch.cuda.device_count()
+torch.cuda.set_device(device)
+
+
+def init_comm(ctx, comm_dir, n, me, job_ranks=None):
+    if transport == "ipc":
+        ctx.comm_init_ipc(comm_dir, n, me, job_ranks)
+    else:                                           # NCCL: comm rank 0 publishes the unique id
+        uid_path = comm_dir + ".uid"
+        if me == 0:
+            open(uid_path + ".tmp", "wb").write(J.get_unique_id())
+            os.rename(uid_path + ".tmp", uid_path)
+        t0 = time.time()
+        while not os.path.exists(uid_path) and time.time() - t0 < 120:
+            time.sleep(0.01)
+        ctx.comm_init(open(uid_path, "rb").read(), n, me, job_ranks)
+
+
+def make_ctx(comm_dir, scramble, comm=True):
+    ctx = J.Context(device=device, rank=rank, world=world, chunk_bytes=1 << 20, image_dir=shm + "/img",
                     staging_bytes=48 << 20, slot_bytes=4 << 20, flags=J.F_TIME_KERNELS)
     sts = {{}}
     for g in groups:
         members = g.members if g.group == 2 else list(range(world))
         if rank in members:
-            st = GroupState(g, seed, fill=not scramble, shuffle_seed=10 * rank + (7 if scramble else 0))
+            st = GroupState(g, seed, device=device, fill=not scramble, shuffle_seed=10 * rank + (7 if scramble else 0))
             if scramble:
                 st.scramble()
             sts[g.group] = st
@@ -54,17 +74,8 @@ def make_ctx(comm_dir, scramble):
             ctx.mark(g.group, 33, J.CLEAN)
         else:
             ctx.declare_group(g.group, g.policy, members)
-    if transport == "ipc":
-        ctx.comm_init_ipc(comm_dir, world, rank)
-    else:                                           # NCCL: rank 0 publishes the unique id
-        uid_path = comm_dir + ".uid"
-        if rank == 0:
-            open(uid_path + ".tmp", "wb").write(J.get_unique_id())
-            os.rename(uid_path + ".tmp", uid_path)
-        t0 = time.time()
-        while not os.path.exists(uid_path) and time.time() - t0 < 120:
-            time.sleep(0.01)
-        ctx.comm_init(open(uid_path, "rb").read(), world, rank)
+    if comm:
+        init_comm(ctx, comm_dir, world, rank)
     return ctx, sts
 
 
@@ -123,6 +134,25 @@ elif phase in ("w0", "repl", "dirty"):
         assert gsel[1]["writers"] == [0, 2]
         check(ctx, sts, {{0}})
     print(phase, "ok", flush=True)
+elif phase in ("w_nosel", "repl_nosel"):
+    # rank 1 died; the survivors 0 and 2 fingerprint, exchange and select over
+    # their own (shrunk) communicator; then a fresh replacement joins a new
+    # communicator and restores in PEER mode WITHOUT any selection or blob: it
+    # receives the selection and the writers' digests over the communicator
+    # (SURVEY.md §8(b); PAPER.md:174 copy from a healthy replica)
+    ctx, sts = make_ctx(None, scramble=(phase == "repl_nosel"), comm=False)
+    sel = None
+    if phase == "w_nosel":
+        init_comm(ctx, shm + "/comm4a", 2, {{0: 0, 2: 1}}[rank], [0, 2])
+        allb = ctx.exchange_records(ctx.fingerprint())
+        st_, sel = J.select_consistent_replica(allb, [0, 2])
+        assert st_ == J.OK, J.parse_selection(sel)
+    init_comm(ctx, shm + "/comm4b", world, rank)
+    res = ctx.restore(J.ALL_GROUPS, J.PEER, sel)
+    if phase == "repl_nosel":
+        check(ctx, sts, {{0, 1, 2}})
+        assert res["groups_done"] == 3, res
+    print(phase, "ok", flush=True)
 elif phase in ("writer", "replacement"):
     # rank 1 died; ranks 0 and 2 keep their state, a replacement process joins
     ctx, sts = make_ctx(shm + "/comm2", scramble=(phase == "replacement"))
@@ -150,10 +180,8 @@ ctx.close()
 
 
 def _env(transport, rank):
-    if transport == "ipc":
-        return dict(os.environ)
-    return dict(os.environ, NCCL_HOSTID=f"jitc-test-host-{rank}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
-                NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0", NCCL_DEBUG="WARN")
+    from tests.mp_util import nccl_env
+    return dict(os.environ) if transport == "ipc" else nccl_env("test", rank)
 
 
 def _spawn(shm, world, phases, transport):
@@ -186,6 +214,19 @@ def test_multirank_peer_restore_of_replacement(transport):
     try:
         outs = _spawn(shm, 3, {0: "writer", 1: "replacement", 2: "writer"}, transport)
         assert "peer ok" in outs[1] and "writer ok" in outs[0] and "writer ok" in outs[2], outs
+    finally:
+        shutil.rmtree(shm, ignore_errors=True)
+
+
+@pytest.mark.parametrize("transport", ["ipc", "nccl"])
+def test_peer_restore_replacement_without_selection(transport):
+    """The replacement passes no selection and no blobs to jitc_restore(PEER):
+    the selection comes from the writers over the new communicator."""
+    shm = f"/dev/shm/jitc-ipc-{os.getpid()}-{uuid.uuid4().hex[:8]}"
+    os.makedirs(shm)
+    try:
+        outs = _spawn(shm, 3, {0: "w_nosel", 1: "repl_nosel", 2: "w_nosel"}, transport)
+        assert "repl_nosel ok" in outs[1] and "w_nosel ok" in outs[0] and "w_nosel ok" in outs[2], outs
     finally:
         shutil.rmtree(shm, ignore_errors=True)
 

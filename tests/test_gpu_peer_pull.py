@@ -28,12 +28,15 @@ from paper_conf_eurosys_guptakkvgkrs24_b200 import jitc as J
 from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
 from workloads import configs as W
 rank, world, shm, flip = {rank}, {world}, {shm!r}, {flip}
+import torch as _t
+device = rank % _t.cuda.device_count()
+_t.cuda.set_device(device)
 w = W.scaled(W.c2(), 60000)
-ctx = J.Context(device=0, rank=rank, world=world, chunk_bytes=1 << 20, image_dir=shm, staging_bytes=64 << 20,
+ctx = J.Context(device=device, rank=rank, world=world, chunk_bytes=1 << 20, image_dir=shm, staging_bytes=64 << 20,
                 slot_bytes=16 << 20)
 keep = []
 for g in w.groups:
-    st = GroupState(g, w.seed, shuffle_seed=11 + rank); keep.append(st)
+    st = GroupState(g, w.seed, device=device, shuffle_seed=11 + rank); keep.append(st)
     ctx.register(g.group, g.policy, list(range(world)), st.table(), keepalive=st)
     ctx.mark(g.group, 21, J.CLEAN)
 blob = ctx.fingerprint()
@@ -59,12 +62,15 @@ from paper_conf_eurosys_guptakkvgkrs24_b200 import jitc as J
 from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
 from workloads import configs as W
 rank, world, shm, writers, expect_bad = {rank}, {world}, {shm!r}, {writers}, {expect_bad}
+import torch as _t
+device = rank % _t.cuda.device_count()
+_t.cuda.set_device(device)
 w = W.scaled(W.c2(), 60000)
-ctx = J.Context(device=0, rank=rank, world=world, chunk_bytes=1 << 20, image_dir=shm, staging_bytes=64 << 20,
+ctx = J.Context(device=device, rank=rank, world=world, chunk_bytes=1 << 20, image_dir=shm, staging_bytes=64 << 20,
                 slot_bytes=16 << 20, flags=J.F_TIME_KERNELS)
 sts = {{}}
 for g in w.groups:
-    st = GroupState(g, w.seed, fill=False, shuffle_seed=99); st.scramble(); sts[g.group] = st
+    st = GroupState(g, w.seed, device=device, fill=False, shuffle_seed=99); st.scramble(); sts[g.group] = st
     ctx.register(g.group, g.policy, list(range(world)), st.table(), keepalive=st)
 t0 = time.time()
 while not all(os.path.exists(f"{{shm}}/ready.{{r}}") for r in writers) and time.time() - t0 < 180:

@@ -34,12 +34,15 @@ from paper_conf_eurosys_guptakkvgkrs24_b200 import jitc as J
 from paper_conf_eurosys_guptakkvgkrs24_b200.state import GroupState
 from workloads import configs as W
 rank, shm, transport = {rank}, {shm!r}, {transport!r}
+import torch as _t
+device = rank % _t.cuda.device_count()
+_t.cuda.set_device(device)
 w = W.scaled(W.c2(), 40000, )
-ctx = J.Context(device=0, rank=rank, world=3, chunk_bytes=1 << 20, image_dir=shm + "/img", staging_bytes=48 << 20,
+ctx = J.Context(device=device, rank=rank, world=3, chunk_bytes=1 << 20, image_dir=shm + "/img", staging_bytes=48 << 20,
                 slot_bytes=8 << 20)
 keep = []
 for g in w.groups:
-    st = GroupState(g, w.seed, shuffle_seed=rank); keep.append(st)
+    st = GroupState(g, w.seed, device=device, shuffle_seed=rank); keep.append(st)
     ctx.register(g.group, g.policy, [0, 1, 2], st.table(), keepalive=st)
     ctx.mark(g.group, 50, J.CLEAN)
 torch.cuda.synchronize()
@@ -91,11 +94,9 @@ ctx.close()
 
 
 def _env(transport, r):
+    from tests.mp_util import nccl_env
     env = dict(os.environ, JITC_PEER_DEAD_MS="500")
-    if transport == "nccl":     # one fake host per rank: NCCL accepts three ranks on one GPU (socket transport)
-        env.update(NCCL_HOSTID=f"jitc-wd-host-{r}", NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1",
-                   NCCL_P2P_DISABLE="1", NCCL_SHM_DISABLE="1", NCCL_NVLS_ENABLE="0", NCCL_DEBUG="WARN")
-    return env
+    return env if transport != "nccl" else nccl_env("wd", r, env)
 
 
 @pytest.mark.parametrize("transport", ["ipc", "nccl"])
