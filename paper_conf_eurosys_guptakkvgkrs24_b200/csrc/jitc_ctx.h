@@ -12,6 +12,8 @@
 #include <sys/file.h>
 #include <sys/mman.h>
 #include <sys/stat.h>
+#include <sys/syscall.h>
+#include <ctype.h>
 #include <sys/types.h>
 #include <unistd.h>
 
@@ -72,6 +74,7 @@ struct GroupState {
   // a shared image is pinned as separate registrations of img_reg_piece bytes
   // each (0: one registration); a host<->device copy must not cross one
   uint64_t img_reg_piece = 0;
+  int img_numa_slices = 0;  // slices given a NUMA policy when this rank created the image
   std::vector<uint8_t*> img_regs;
   std::string img_path;
   std::vector<uint8_t> man_priv, commit_priv;  // private-memory manifest / commit

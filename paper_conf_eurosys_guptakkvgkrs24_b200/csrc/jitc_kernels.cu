@@ -344,7 +344,7 @@ int segment_grid(int device) {
 // (CUDA_MODULE_LOADING=LAZY, the default) a kernel's first launch loads its
 // code, and that load waits behind work already running on the device -- e.g.
 // a collective hung on a dead peer -- so a first launch inside the failure
-// path would deadlock (measured: tools/wd_debug*.py).  jitc_create calls this.
+// path would deadlock (measured: tools/debug/wd_debug*.py).  jitc_create calls this.
 cudaError_t preload_kernels() {
   cudaFuncAttributes fa;
   const void* fns[] = {(const void*)seg_kernel<kDigest>, (const void*)seg_kernel<kPack>,

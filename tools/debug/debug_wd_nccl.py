@@ -13,7 +13,7 @@ import textwrap
 import time
 import uuid
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 RANK = r"""
 import faulthandler, os, sys, time
