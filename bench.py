@@ -465,8 +465,17 @@ def run_jitc(args):
         dist.init_process_group("gloo")
 
     w, victim = make_workload(args, world)
-    job = os.environ.get("TORCHELASTIC_RUN_ID", str(os.getpid())) if world > 1 else str(os.getpid())
+    # a fresh directory per run: the IPC transport's control block must never
+    # be a stale one (a crashed earlier run with the same torchrun run id
+    # would leave published IPC handles of dead processes behind)
+    job = [f"{os.getpid()}-{int(time.time() * 1e3) % 10**9}"]
+    if world > 1:
+        dist.broadcast_object_list(job, src=0)
+    job = job[0]
     shm = args.image_dir or f"/dev/shm/jitc-bench-{job}"
+    if rank == 0 and not args.image_dir:   # also on an exception: never leave a 128 GB image behind
+        import atexit
+        atexit.register(lambda: [shutil.rmtree(d, ignore_errors=True) for d in (shm, f"{shm}-comm", f"{shm}-comm2")])
     flags = J.F_TIME_KERNELS
     if args.zero_copy:
         flags |= J.F_ZERO_COPY_D2H | J.F_ZERO_COPY_H2D

@@ -53,7 +53,7 @@
 extern "C" {
 #endif
 
-#define JITC_ABI_VERSION 1
+#define JITC_ABI_VERSION 2  /* 2: jitc_stats.groups_done / groups_skipped, timeline spans */
 #define JITC_ALL_GROUPS 0xFFFFFFFFu
 
 typedef struct jitc_ctx jitc_ctx;
@@ -445,6 +445,28 @@ jitc_status jitc_waste_model(int32_t kind, double n_gpus, double f, double o, do
 /* ---- counters ---------------------------------------------------------------- */
 jitc_status jitc_kernel_counters(jitc_ctx* ctx, int32_t kind, jitc_kernel_counter* out);
 jitc_status jitc_reset_counters(jitc_ctx* ctx);
+
+/* ---- timeline (overlap evidence; nsys is not available on the boxes) --------- */
+/* One span of work on a library stream: a kernel launch (kind 1 K1, 2 K2,
+ * 3 K3, 4 K5), a copy-engine transfer batch (10 D2H, 11 H2D, 12 peer copy)
+ * of one pipeline round.  t0/t1 are CUDA-event times in ms relative to the
+ * jitc_timeline_start event; stream 0 = compute, 1 = copy. */
+typedef struct {
+    int32_t kind;
+    int32_t stream;
+    uint32_t group;
+    uint32_t round;
+    double t0_ms, t1_ms;
+    uint64_t bytes;
+} jitc_span;
+/* Starts recording spans of the following calls (up to max_spans; events are
+ * created here, in steady state).  Each span costs two timing-event records
+ * (~40 us each next to a copy-engine transfer), so this is a
+ * diagnostic, not the bench's timed configuration. */
+jitc_status jitc_timeline_start(jitc_ctx* ctx, uint32_t max_spans);
+/* Stops recording and writes up to cap spans (after the recorded calls
+ * returned); *n = spans recorded.  cap == 0 => only *n. */
+jitc_status jitc_timeline_read(jitc_ctx* ctx, jitc_span* out, size_t cap, size_t* n);
 
 /* ---- test/bench harness kernels (K4; not part of the method) ------------- */
 /* Fills numel elements of a device tensor with the O9 counter-based generator

@@ -46,6 +46,7 @@ static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelectio
         int sl = (int)(j % nslots);
         uint8_t* slot = c->staging + sl * R;
         if (j >= (uint32_t)nslots) CU(cudaStreamWaitEvent(c->s_comp, c->ev_free[sl], 0));
+        c->tl_group = g.id, c->tl_round = j;
         uint32_t lo, hi;
         seg_span(g, a, b, &lo, &hi);
         jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, slot, a), g.d_dig2, b - a);
@@ -158,6 +159,7 @@ static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection
     while (e < ops.size() && ops[e].round == j) ++e;
     const uint32_t sl = j % S;
     const uint64_t seq = (gen << 24) | (j + 1);
+    c->tl_group = g.id, c->tl_round = j;
     if (e > i) ++rounds;
     if (e > i && used[sl]) CU(cudaStreamWaitEvent(c->s_comp, c->ev_free[sl], 0));
     bool packs = false;
@@ -190,8 +192,10 @@ static jitc_status fanout_group(jitc_ctx* c, GroupState& g, const GroupSelection
         recv = true;
         jitc_status st = ipc_wait_peer(*ic, op.peer, &ic->ctl->cap_posted[ic->slot[op.peer]][gsl], seq, "a writer to post a round");
         if (st) return st;
+        const size_t tl0 = tl_open(c, c->s_comp);
         CU(cudaMemcpyAsync(c->staging + op.off, ic->peer_staging[op.peer] + op.off, op.bytes, cudaMemcpyDefault,
                            c->s_comp));
+        tl_close(c, tl0, c->s_comp, 12, op.bytes);
         if (stats) stats->p2p_bytes += op.bytes;
       }
       if (recv || is_mover) {

@@ -18,6 +18,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <functional>
 #include <chrono>
 #include <atomic>
 #include <condition_variable>
@@ -215,6 +216,19 @@ struct jitc_ctx {
   // test hook (JITC_DEBUG_FP_PAUSE_US, read at create): pause between the end
   // of K1 and the second phase-word read of jitc_fingerprint (seqlock test)
   uint32_t debug_fp_pause_us = 0;
+  // timeline (jitc_timeline_start / _read): two timing events per span
+  struct TlRec {
+    int32_t kind, stream;
+    uint32_t group, round;
+    uint64_t bytes;
+    size_t e0, e1;
+  };
+  bool tl_on = false;
+  std::vector<cudaEvent_t> tl_ev;
+  std::vector<TlRec> tl;
+  size_t tl_ev_used = 0;
+  cudaEvent_t tl_base = nullptr;
+  uint32_t tl_group = 0, tl_round = 0;  // attribution of the spans being recorded
   // counters
   jitc_kernel_counter kc[5]{};
   uint64_t launches_in_call = 0;
@@ -263,10 +277,25 @@ struct NvtxRange {
   ~NvtxRange() { nvtxRangePop(); }
 };
 
+// Timeline spans (jitc_timeline_start): tl_open records the start event on
+// stream s and returns its index (or SIZE_MAX when off / full); tl_close
+// records the end event and the span.
+inline size_t tl_open(jitc_ctx* c, cudaStream_t s) {
+  if (!c->tl_on || c->tl_ev_used + 2 > c->tl_ev.size()) return SIZE_MAX;
+  if (cudaEventRecord(c->tl_ev[c->tl_ev_used], s) != cudaSuccess) return SIZE_MAX;
+  return c->tl_ev_used++;
+}
+inline void tl_close(jitc_ctx* c, size_t e0, cudaStream_t s, int kind, uint64_t bytes) {
+  if (e0 == SIZE_MAX || c->tl_ev_used + 1 > c->tl_ev.size()) return;
+  if (cudaEventRecord(c->tl_ev[c->tl_ev_used], s) != cudaSuccess) return;
+  c->tl.push_back({kind, s == c->s_copy ? 1 : 0, c->tl_group, c->tl_round, bytes, e0, c->tl_ev_used++});
+}
+
 // Kernel launch with optional event bracketing (JITC_F_TIME_KERNELS).
 inline jitc_status run_segments(jitc_ctx* c, GroupState& g, int mode, const LaunchRanges& r, uint64_t* dig,
                          uint64_t bytes, const uint64_t* remote = nullptr) {
   bool timed = (c->cfg.flags & JITC_F_TIME_KERNELS) && c->kev_used + 2 <= c->kev.size();
+  const size_t tl0 = tl_open(c, c->s_comp);
   if (timed) CU(cudaEventRecord(c->kev[c->kev_used], c->s_comp));
   CU(launch_segments(mode, g.d_segs, r, dig, c->grid, c->d_work, c->s_comp, remote,
                      timed && c->d_span ? c->d_span + c->kev_used : nullptr));
@@ -276,6 +305,7 @@ inline jitc_status run_segments(jitc_ctx* c, GroupState& g, int mode, const Laun
     c->kev_bytes[c->kev_used / 2] = bytes;
     c->kev_used += 2;
   }
+  tl_close(c, tl0, c->s_comp, mode, bytes);
   c->launches_in_call++;
   c->kc[mode].launches++;
   c->kc[mode].bytes += bytes;
@@ -318,8 +348,9 @@ inline void finish_stats(jitc_ctx* c, const CallTimer& t, jitc_stats* st, bool d
 // memory `dev`, issued in pieces of at most c->copy_piece bytes that never
 // cross a registration boundary of the pinned image (cudaMemcpy refuses a
 // host range that spans two registrations).
-inline cudaError_t copy_image(const jitc_ctx* c, const GroupState& g, uint64_t img_off, void* dev, uint64_t n,
+inline cudaError_t copy_image(jitc_ctx* c, const GroupState& g, uint64_t img_off, void* dev, uint64_t n,
                               cudaMemcpyKind kind, cudaStream_t s) {
+  const size_t tl0 = tl_open(c, s);
   const uint64_t P = c->copy_piece ? c->copy_piece : n;
   const uint64_t R = g.img_reg_piece;
   uint64_t o = 0;
@@ -333,6 +364,7 @@ inline cudaError_t copy_image(const jitc_ctx* c, const GroupState& g, uint64_t i
     if (e != cudaSuccess) return e;
     o += len;
   }
+  tl_close(c, tl0, s, kind == cudaMemcpyDeviceToHost ? 10 : 11, n);
   return cudaSuccess;
 }
 

@@ -105,6 +105,7 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
     while (e < ops.size() && ops[e].round == j && ops[e].kind != kOpDigestSend && ops[e].kind != kOpDigestRecv) ++e;
     const uint32_t sl = j % (S ? S : 1);
     const uint64_t seq = base_round + j + 1;  // IPC: this round's counter value
+    c->tl_group = g.id, c->tl_round = j;
     bool writes_slot = false;
     for (size_t q = i; q < e; ++q) writes_slot |= ops[q].kind == kOpH2D || ops[q].kind == kOpPack;
     if (e > i) ++rounds;
@@ -308,6 +309,7 @@ static jitc_status restore_peer(jitc_ctx* c, GroupState& g, const GroupSelection
   jitc_status st = make_plan(c, in, &ops, &S, &J);
   if (st) return st;
   if (!is_writer && !is_dst) return JITC_OK;
+  if (in.dests.empty()) return JITC_OK;  // every member is a writer: nobody to rebuild (the plan is empty)
   // 1. the lowest writer sends the selected class's digests to every destination
   uint64_t* d_expect = g.d_dig;
   if (is_writer && (!g.has_fp || g.fp_root != gs.root))

@@ -65,12 +65,22 @@ class Stats(ctypes.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class Span(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("stream", ctypes.c_int32), ("group", ctypes.c_uint32),
+                ("round", ctypes.c_uint32), ("t0_ms", ctypes.c_double), ("t1_ms", ctypes.c_double),
+                ("bytes", ctypes.c_uint64)]
+
+
+SPAN_KIND = {1: "K1", 2: "K2", 3: "K3", 4: "K5", 10: "D2H", 11: "H2D", 12: "P2P"}
+
+
 class KernelCounter(ctypes.Structure):
     _fields_ = [("launches", ctypes.c_uint64), ("bytes", ctypes.c_uint64), ("ms", ctypes.c_double),
                 ("span_ms", ctypes.c_double)]
 
 
 _lib = None
+ABI_VERSION = 2   # include/jitc.h JITC_ABI_VERSION
 
 
 def lib() -> ctypes.CDLL:
@@ -82,6 +92,8 @@ def lib() -> ctypes.CDLL:
         raise RuntimeError(f"{SO_PATH} not built: run `python -m paper_conf_eurosys_guptakkvgkrs24_b200.build` "
                            "(there is no CPU fallback)")
     L = ctypes.CDLL(SO_PATH)
+    if L.jitc_abi_version() != ABI_VERSION:
+        raise RuntimeError(f"{SO_PATH} has ABI {L.jitc_abi_version()}, this binding expects {ABI_VERSION}: rebuild it")
     i32, u32, u64, vp, sz = ctypes.c_int32, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_size_t
     P = ctypes.POINTER
     sig = {
@@ -115,6 +127,8 @@ def lib() -> ctypes.CDLL:
         "jitc_attach_image": ([vp, u32, u64], i32),
         "jitc_kernel_counters": ([vp, i32, P(KernelCounter)], i32),
         "jitc_reset_counters": ([vp], i32),
+        "jitc_timeline_start": ([vp, u32], i32),
+        "jitc_timeline_read": ([vp, P(Span), sz, P(sz)], i32),
         "jitc_gen_fill": ([vp, u32, u64, u64, u32, u32, u32, u32, i32, vp], i32),
         "jitc_inject_update": ([vp, u64, u64, u32, u64, vp], i32),
         "jitc_inject_rne": ([vp, vp, u64, vp], i32),
@@ -151,7 +165,7 @@ EXPORTED = ["jitc_create", "jitc_destroy", "jitc_last_error", "jitc_abi_version"
             "jitc_inject_update", "jitc_inject_rne", "jitc_inject_bitflip", "jitc_inject_hang",
             "jitc_inject_release", "jitc_capture_local", "jitc_set_aux", "jitc_get_aux", "jitc_peer_export", "jitc_restore_pull", "jitc_persist", "jitc_stage_in", "jitc_waste_model", "jitc_watch_event", "jitc_watchdog_start", "jitc_watchdog_wait",
             "jitc_watchdog_stop", "jitc_watchdog_failed", "jitc_capture_plan", "jitc_capture_fanout",
-            "jitc_attach_image", "jitc_liveness_init", "jitc_comm_dead"]
+            "jitc_attach_image", "jitc_liveness_init", "jitc_comm_dead", "jitc_timeline_start", "jitc_timeline_read"]
 ON_HANG_NOTIFY, ON_HANG_LOCAL_CAPTURE, ON_HANG_COLLECTIVE_CAPTURE = 0, 1, 2
 
 
@@ -510,6 +524,18 @@ class Context:
         kc = KernelCounter()
         _check(self._L.jitc_kernel_counters(self._h, kind, ctypes.byref(kc)), "jitc_kernel_counters")
         return dict(launches=kc.launches, bytes=kc.bytes, ms=kc.ms, span_ms=kc.span_ms)
+
+    def timeline_start(self, max_spans: int = 4096):
+        """Record the spans (kernel launches, copy batches) of the following calls."""
+        _check(self._L.jitc_timeline_start(self._h, max_spans), "jitc_timeline_start")
+
+    def timeline_read(self) -> list:
+        n = ctypes.c_size_t()
+        _check(self._L.jitc_timeline_read(self._h, None, 0, ctypes.byref(n)), "jitc_timeline_read")
+        buf = (Span * max(n.value, 1))()
+        _check(self._L.jitc_timeline_read(self._h, buf, n.value, ctypes.byref(n)), "jitc_timeline_read")
+        return [dict(kind=SPAN_KIND.get(x.kind, x.kind), stream=x.stream, group=x.group, round=x.round,
+                     t0_ms=x.t0_ms, t1_ms=x.t1_ms, bytes=x.bytes) for x in buf[:n.value]]
 
     def reset_counters(self):
         _check(self._L.jitc_reset_counters(self._h), "jitc_reset_counters")

@@ -30,7 +30,7 @@ def test_exports_every_declared_symbol(J):
     for name in declared:
         assert hasattr(L, name), name
     assert set(J.EXPORTED) == declared
-    assert L.jitc_abi_version() == 1
+    assert L.jitc_abi_version() == 2
 
 
 def test_no_cpu_fallback(J):

@@ -32,10 +32,11 @@ def test_bench_two_ranks_one_gpu(transport):
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
-    assert d["n_gpus"] == 2 and d["config"]["writers_k"] == 2 and d["config"]["transport"] == transport
+    assert d["n_gpus"] == 2 and d["config"]["writers_k"] == {"0": 2} and d["config"]["transport"] == transport
     assert d["value"] > 0 and d["gpu_launches"] > 0
     pr = d["peer_restore"]           # the last rank rebuilt from the other's live HBM (PEER mode)
-    assert pr["replacement"] == 1 and pr["writers"] == 1 and pr["replacement_ingress_bytes"] == d["config"]["image_bytes"]
+    assert pr["replacement"] == 1 and pr["writers_k"] == {"0": 1} and not pr["replacement_passed_selection"]
+    assert pr["replacement_ingress_bytes"] == d["config"]["image_bytes"]
 
 
 def test_bench_n1_json_contract():
