@@ -163,6 +163,8 @@ jitc_status jitc_create(const jitc_config* cfg, jitc_ctx** out) {
   cudaGetLastError();
   c->grid = segment_grid(c->device);
   if (const char* e = getenv("JITC_DEBUG_FP_PAUSE_US")) c->debug_fp_pause_us = (uint32_t)strtoul(e, nullptr, 10);
+  if (const char* e = getenv("JITC_DEBUG_EXIT_AFTER_ROUND"))
+    c->debug_exit_after_round = (uint32_t)strtoul(e, nullptr, 10);
   *out = c.release();
   return JITC_OK;
 }

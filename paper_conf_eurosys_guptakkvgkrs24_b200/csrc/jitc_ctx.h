@@ -216,6 +216,10 @@ struct jitc_ctx {
   // test hook (JITC_DEBUG_FP_PAUSE_US, read at create): pause between the end
   // of K1 and the second phase-word read of jitc_fingerprint (seqlock test)
   uint32_t debug_fp_pause_us = 0;
+  // test hook (JITC_DEBUG_EXIT_AFTER_ROUND=j, read at create): with the IPC
+  // transport, the process exits right after posting restore round j - 1, so
+  // that its peers' restore aborts part-way (tests/test_gpu_writer_death.py)
+  uint32_t debug_exit_after_round = 0;
   // timeline (jitc_timeline_start / _read): two timing events per span
   struct TlRec {
     int32_t kind, stream;

@@ -142,6 +142,11 @@ static jitc_status execute_plan(jitc_ctx* c, GroupState& g, const std::vector<Pl
     if (ic) {
       jitc_status st = ipc_post(c, &ic->ctl->posted[my_slot][gs], seq, c->s_comp);  // my block is ready
       if (st) return st;
+      if (c->debug_exit_after_round && j + 1 >= c->debug_exit_after_round) {
+        cudaStreamSynchronize(c->s_comp);
+        cudaStreamSynchronize(c->s_copy);
+        _exit(17);
+      }
       for (size_t q = i; q < e; ++q) {
         const PlanOp& op = ops[q];
         if (op.kind != kOpUnpack || op.peer == c->comm_rank) continue;

@@ -168,3 +168,68 @@ def test_writer_dies_during_peer_restore_no_hang(transport):
         assert procs[0].returncode == 0 and "rank 0 " in outs[0], "\n=====\n".join(outs)
     finally:
         shutil.rmtree(shm, ignore_errors=True)
+
+
+RETRY_RANK = RANK.split("allb = ctx.exchange_records(ctx.fingerprint())")[0] + r"""
+import numpy as np
+from oracle import oracle as O
+allb = ctx.exchange_records(ctx.fingerprint())
+s_, sel = J.select_consistent_replica(allb, [0, 1, 2])
+assert s_ == J.OK
+ctx.capture(sel)
+ctx.commit(sel)                                    # a complete 3-way checkpoint
+for st in keep:
+    st.scramble()
+t0 = time.time()
+try:                                               # rank 2 exits part-way through (JITC_DEBUG_EXIT_AFTER_ROUND)
+    ctx.restore(J.ALL_GROUPS, J.HOST)
+    raise SystemExit("restore completed without rank 2")
+except J.JitcError as e:
+    assert e.status == J.EPEER, e
+dead = ctx.comm_dead()
+while not dead and time.time() - t0 < 10:
+    time.sleep(0.05)
+    dead = ctx.comm_dead()
+assert dead == [2], dead
+ctx.comm_shrink(dead)
+res = ctx.restore(J.ALL_GROUPS, J.HOST)            # retry: 2-way slices, fresh round generation
+for g in w.groups:
+    ctx.verify(g.group)
+torch.cuda.synchronize()
+for st, g in zip(keep, w.groups):
+    for i, t in enumerate(g.tensors):
+        assert np.array_equal(st.tensor_bytes(i).cpu().numpy(), O.gen_tensor_bytes(t, w.seed, g.group)), t.name
+print("survivor", rank, "retried restore bit-exact in", res["rounds"], "rounds", flush=True)
+ctx.close()
+"""
+
+
+def test_restore_aborted_part_way_then_retried():
+    """ADVICE r01 (IPC restore rounds): a rank dies after posting its first
+    rounds of a 3-way HOST restore, so the survivors' restore aborts with
+    JITC_EPEER part-way, with the shared round counters already advanced.  The
+    survivors shrink and retry the restore 2-way: every call has its own round
+    generation, so no wait can pass on a stale counter of the aborted call, and
+    the retry is bit-exact against the oracle."""
+    shm = f"/dev/shm/jitc-rretry-{os.getpid()}-{uuid.uuid4().hex[:8]}"
+    os.makedirs(shm)
+    try:
+        procs = []
+        for r in range(3):
+            env = _env("ipc", r)
+            if r == 2:
+                env["JITC_DEBUG_EXIT_AFTER_ROUND"] = "2"
+            procs.append(subprocess.Popen([sys.executable, "-c", textwrap.dedent(RETRY_RANK.format(
+                root=ROOT, rank=r, shm=shm, transport="ipc"))], cwd=ROOT, stdout=subprocess.PIPE,
+                stderr=subprocess.STDOUT, text=True, env=env))
+        try:
+            outs = [p.communicate(timeout=300)[0] for p in procs]
+        finally:
+            for p in procs:
+                if p.poll() is None:
+                    p.kill()
+        assert procs[2].returncode == 17, "\n=====\n".join(outs)
+        for i in (0, 1):
+            assert procs[i].returncode == 0 and "retried restore bit-exact" in outs[i], "\n=====\n".join(outs)
+    finally:
+        shutil.rmtree(shm, ignore_errors=True)
