@@ -15,7 +15,7 @@ namespace jitc {
 
 constexpr uint64_t kGolden = 0x9E3779B97F4A7C15ull;  // JF64 key step (2^64 / golden ratio)
 constexpr uint64_t kAlign = 256;                       // image alignment (reading R4)
-constexpr uint32_t kMaxSegBytes = 32u << 10;           // K1/K2/K3 work unit (data bytes)
+constexpr uint32_t kMaxSegBytes = 128u << 10;          // K1/K2/K3 work unit (data bytes)
 constexpr int kMaxPhaseSlots = 512;
 constexpr int kEventPool = 8192;
 
@@ -72,6 +72,8 @@ struct LaunchRanges {
 // d_work: 2 x u32 zero-initialised device counters, private to the stream
 // (the kernel resets them when it finishes).
 // d_remote (kPull only): per-segment source address in a peer's memory.
+// grid: the device's SM count (segment_grid); each mode launches that many
+// times its own resident CTAs per SM (jitc_kernels.cu, "CTA shape per mode").
 cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, uint64_t* d_dig, int grid,
                             uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote,
                             unsigned long long* d_span = nullptr);

@@ -17,19 +17,32 @@
 // wrap-around sum of its terms.  The sum is order-free, so every CTA adds its
 // partial into d[chunk] with a 64-bit atomic and the result is deterministic.
 //
-// Work unit: one Seg = one piece (<= 32 KiB) of one tensor that never crosses
-// a chunk boundary.  CTAs of a persistent grid grab batches of 8 consecutive
-// segments from an atomic counter; inside a segment every thread streams 16-byte vectors (4 loads in flight before
-// any use), hashes both words, optionally stores, and the warp reduces its
+// Work unit: one Seg = one piece (<= 128 KiB) of one tensor that never crosses
+// a chunk boundary.  CTAs of a persistent grid grab batches of consecutive
+// segments from an atomic counter; inside a segment every thread streams 16-byte vectors (4 or 8 loads in flight
+// before any use), hashes both words, optionally stores, and the warp reduces its
 // partial with shuffles before one atomicAdd per warp per chunk it touched.  Pure HBM
 // (or PCIe) streaming: no tensor cores, no shared-memory reuse (every byte is
 // touched once), so the design targets coalescing, MLP and a grid sized to
 // the SM count.
+//
+// CTA shape per mode (round 2, tools/k2_variants.cu sweeps on B200,
+// profiles/r02c_k2_variants.txt).  Work grabs of 128-256 KiB and enough loads
+// in flight per SM are what matter; the per-segment bookkeeping (descriptor,
+// range lookup, tail test) is amortised over 128 KiB segments:
+//  * read+write kernels (K2, K3, K5): 512 threads x 4 vectors (32 KiB per
+//    unrolled step), 2 CTAs per SM, one segment per grab.  6.84 TB/s vs
+//    6.29 TB/s for round 1's 256-thread, 8-CTA, 32-register shape with 32 KiB
+//    segments on the same box (a D2D cudaMemcpy: 6.5-6.6 TB/s);
+//  * read-only K1: 256 threads x 8 vectors, 4 CTAs per SM, two segments per
+//    grab: 7.34 vs 6.83 TB/s; with no stores in flight it needs more loads
+//    per thread to cover the read latency.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
 #include <string.h>
 
+#include <atomic>
 #include <string>
 
 #include "jitc_internal.h"
@@ -38,8 +51,12 @@ namespace jitc {
 
 namespace {
 
-constexpr int kThreads = 256;
-constexpr int kUnroll = 4;
+// threads per CTA, vectors in flight per thread, resident CTAs per SM (the
+// register budget given to ptxas: without it ptxas picks 32 registers and
+// serialises the loads of a step), and segments per work grab, by mode
+// (see the header)
+template <int MODE> struct Shape { static constexpr int T = 512, U = 4, MINB = 2, B = 1; };
+template <> struct Shape<kDigest> { static constexpr int T = 256, U = 8, MINB = 4, B = 2; };
 constexpr uint64_t PHI = 0x9E3779B97F4A7C15ull;
 
 __device__ __forceinline__ uint64_t dmix(uint64_t x) {
@@ -51,14 +68,22 @@ __device__ __forceinline__ uint64_t dmix(uint64_t x) {
   return x;
 }
 
+// Loads are asm volatile so that all kUnroll loads of a step issue before
+// the hashing that consumes them (measured +1-2% over letting ptxas interleave).
 __device__ __forceinline__ uint4 ld_stream(const uint4* p) {
   uint4 v;
-  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
                : "l"(p));
   return v;
 }
-__device__ __forceinline__ uint4 ld_plain(const uint4* p) { return __ldcs(p); }
+__device__ __forceinline__ uint4 ld_plain(const uint4* p) {
+  uint4 v;
+  asm volatile("ld.global.cs.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p));
+  return v;
+}
 __device__ __forceinline__ void st_stream(uint4* p, uint4 v) { __stcs(p, v); }
 __device__ __forceinline__ uint64_t lo64(uint4 v) { return (uint64_t)v.x | ((uint64_t)v.y << 32); }
 __device__ __forceinline__ uint64_t hi64(uint4 v) { return (uint64_t)v.z | ((uint64_t)v.w << 32); }
@@ -109,15 +134,13 @@ __device__ __forceinline__ void flush(unsigned long long* dig, uint32_t chunk, u
   if (lane == 0) atomicAdd(dig + chunk, (unsigned long long)acc);
 }
 
-// Dynamic work distribution: CTAs grab batches of kBatch consecutive
+// Dynamic work distribution: CTAs grab batches of Shape<MODE>::B consecutive
 // segments (<= 256 KiB) from a global counter, so SMs that stream faster take
 // more work and no CTA idles at the tail.  Inside a batch the next
 // descriptor is prefetched while the current segment streams, and the
 // partial digest stays in registers until the chunk changes.  The counter
 // pair (next batch, finished CTAs) resets itself: the last CTA to finish
 // zeroes it for the next launch on the stream.
-constexpr uint32_t kBatch = 8;
-
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -128,11 +151,14 @@ __device__ __forceinline__ unsigned long long gtimer() {
 // ~(first CTA start), span[1] = last CTA end, in %globaltimer nanoseconds
 // (the start is stored inverted so that both ends are an atomicMax).
 template <int MODE>
-__global__ void __launch_bounds__(kThreads) seg_kernel(const Seg* __restrict__ segs, LaunchRanges R,
+__global__ void __launch_bounds__(Shape<MODE>::T, Shape<MODE>::MINB) seg_kernel(const Seg* __restrict__ segs, LaunchRanges R,
                                                        unsigned long long* __restrict__ dig,
                                                        unsigned int* __restrict__ work,
                                                        const uint64_t* __restrict__ remote,
                                                        unsigned long long* __restrict__ span) {
+  constexpr int kThreads = Shape<MODE>::T;
+  constexpr int kUnroll = Shape<MODE>::U;
+  constexpr uint32_t kBatch = Shape<MODE>::B;
   if (span && threadIdx.x == 0) atomicMax(span, ~gtimer());
   const uint32_t total = R.prefix[R.n];
   const uint32_t nbatch = (total + kBatch - 1) / kBatch;
@@ -324,20 +350,37 @@ __global__ void release_kernel(uint32_t* flag, uint32_t v) {
 uint32_t* g_hang_d = nullptr;  // 64 device release flags
 cudaStream_t g_hang_s = nullptr;
 
-int g_grid[64] = {0};
+// Computed once, read by every launch (any thread: the watchdog's action
+// launches too), hence atomics; a racing first computation stores the same value.
+std::atomic<int> g_sms[64];
+std::atomic<int> g_per[8];  // resident CTAs per SM, by mode
+
+template <int MODE>
+int per_sm() {
+  int v = g_per[MODE].load(std::memory_order_relaxed);
+  if (!v) {
+    int per = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, seg_kernel<MODE>, Shape<MODE>::T, 0);
+    v = per > 0 ? per : 1;
+    g_per[MODE].store(v, std::memory_order_relaxed);
+  }
+  return v;
+}
 
 }  // namespace
 
+// SM count of the device; launch_segments sizes each mode's persistent grid
+// as this x the mode's resident CTAs per SM.
 int segment_grid(int device) {
-  if (device < 0 || device >= 64) return 148 * 8;
-  if (!g_grid[device]) {
-    int sms = 148, per = 0;
+  if (device < 0 || device >= 64) return 148;
+  int v = g_sms[device].load(std::memory_order_relaxed);
+  if (!v) {
+    int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, seg_kernel<kPack>, kThreads, 0);
-    if (per <= 0) per = 4;
-    g_grid[device] = sms * per;
+    v = sms > 0 ? sms : 148;
+    g_sms[device].store(v, std::memory_order_relaxed);
   }
-  return g_grid[device];
+  return v;
 }
 
 // Force-load every kernel of this module.  With CUDA lazy loading
@@ -380,16 +423,29 @@ cudaError_t launch_segments(int mode, const Seg* d_segs, const LaunchRanges& r, 
                             uint32_t* d_work, cudaStream_t s, const uint64_t* d_remote, unsigned long long* d_span) {
   uint32_t total = r.prefix[r.n];
   if (total == 0) return cudaSuccess;
-  uint32_t nbatch = (total + kBatch - 1) / kBatch;
-  int g = (int)(nbatch < (uint32_t)grid ? nbatch : (uint32_t)grid);
   auto* dig = reinterpret_cast<unsigned long long*>(d_dig);
+  // grid = SMs x resident CTAs of this mode, or fewer when there are fewer batches
+  auto size = [&](int per, uint32_t batch) {
+    uint32_t nbatch = (total + batch - 1) / batch, full = (uint32_t)grid * (uint32_t)per;
+    return (int)(nbatch < full ? nbatch : full);
+  };
   switch (mode) {
-    case kDigest: seg_kernel<kDigest><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr, d_span); break;
-    case kPack: seg_kernel<kPack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr, d_span); break;
-    case kUnpack: seg_kernel<kUnpack><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, nullptr, d_span); break;
+    case kDigest:
+      seg_kernel<kDigest><<<size(per_sm<kDigest>(), Shape<kDigest>::B), Shape<kDigest>::T, 0, s>>>(
+          d_segs, r, dig, d_work, nullptr, d_span);
+      break;
+    case kPack:
+      seg_kernel<kPack><<<size(per_sm<kPack>(), Shape<kPack>::B), Shape<kPack>::T, 0, s>>>(d_segs, r, dig, d_work,
+                                                                                          nullptr, d_span);
+      break;
+    case kUnpack:
+      seg_kernel<kUnpack><<<size(per_sm<kUnpack>(), Shape<kUnpack>::B), Shape<kUnpack>::T, 0, s>>>(
+          d_segs, r, dig, d_work, nullptr, d_span);
+      break;
     case kPull:
       if (!d_remote) return cudaErrorInvalidValue;
-      seg_kernel<kPull><<<g, kThreads, 0, s>>>(d_segs, r, dig, d_work, d_remote, d_span);
+      seg_kernel<kPull><<<size(per_sm<kPull>(), Shape<kPull>::B), Shape<kPull>::T, 0, s>>>(d_segs, r, dig, d_work,
+                                                                                          d_remote, d_span);
       break;
     default: return cudaErrorInvalidValue;
   }
