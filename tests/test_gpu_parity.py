@@ -166,6 +166,50 @@ def test_capture_restore_bit_exact(J, shm, flags, C):
         ctx.close()
 
 
+def _segment_edge_table():
+    """Tensors whose sizes straddle the kernels' 128 KiB segment (work unit)
+    and the 64 KiB / 1 MiB chunks: every piece shape K1/K2/K3 cut a tensor
+    into (whole segments, a ragged last segment, a < 16-B data tail, pieces
+    ended by a chunk edge), with vector and scalar paths via misalignment."""
+    K = 1 << 17
+    g = W.GroupSpec(11, W.REQUIRED, [0])
+    sizes = [K - 16, K - 1, K, K + 1, K + 8, K + 16, K + 17, 2 * K + 3, (1 << 20) - 1, (1 << 20) + 5,
+             3 * (1 << 20) + 7, 40000, 5]
+    for i, b in enumerate(sizes):
+        g.tensors.append(W.TensorSpec(f"u{i}", "u8", b, "bytes", i))
+    g.tensors.append(W.TensorSpec("f", "f32", 300_001, "master", 100))
+    g.tensors.append(W.TensorSpec("h", "bf16", 200_001, "grad", 101))
+    g.tensors.append(W.TensorSpec("z", "zeros", K + 3, "bytes", 102))
+    return g
+
+
+@pytest.mark.parametrize("C", [1 << 16, 1 << 20])
+@pytest.mark.parametrize("misalign", [0, 1, 2, 8])
+def test_segment_boundaries_bit_exact(J, shm, C, misalign):
+    """K1 digests, the K2 image, the K3 restore and A12 verify equal the oracle
+    on tensors cut at every kind of segment / chunk boundary (round-2 128 KiB
+    segments, 512-thread read+write CTAs, 8-load K1)."""
+    g = _segment_edge_table()
+    st = _state(g, 77, misalign=misalign)
+    ctx = _ctx(J, C, image_dir=shm, staging=8 * C * 4, slot=4 * C)
+    lh, L = ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+    lay = O.layout_of_group(g, C)
+    assert (lh, L) == (lay.layout_hash, lay.L)
+    ctx.mark(g.group, 9, J.CLEAN)
+    blob, sel, cap = _pipeline(J, ctx)
+    want = O.pack(O.gen_group(g, 77), lay)
+    assert np.array_equal(_records(blob)[g.group].d, O.jf64(want, C, 0, lay.n_c))
+    img = np.fromfile(f"{shm}/g{g.group}.img", dtype=np.uint8)[:lay.L]
+    assert np.array_equal(img, want)
+    st.scramble()
+    ctx.restore(g.group, J.HOST)
+    torch.cuda.synchronize()
+    for i, t in enumerate(g.tensors):
+        assert np.array_equal(st.tensor_bytes(i).cpu().numpy(), O.gen_tensor_bytes(t, 77, g.group)), t.name
+    assert ctx.verify(g.group, blob) == 2**64 - 1
+    ctx.close()
+
+
 @pytest.mark.parametrize("flags", [0, 3])
 @pytest.mark.parametrize("piece_mb", [1, 3])
 def test_capture_restore_image_pinned_in_pieces(J, shm, monkeypatch, flags, piece_mb):
