@@ -327,11 +327,14 @@ def cpu_baseline(w, rank: int, blob: bytes, committed: dict, digests: dict, ever
     one = rec1.run(1, blob=blob, digests=digests)
     wall = time.perf_counter() - t0
     return {"value": full["GBps"], "unit": "GB/s", "cores": nth, "kind": "oracle",
-            "sample": f"{w.name}: whole replica ({rec1.L / 1e9:.2f} GB); JF64 over the committed /dev/shm image "
-                      f"(every chunk, checked against the K1 digests); pack and unpack+verify on 1/{every} of the "
-                      f"chunks, evenly spaced, extrapolated by bytes; {nth} threads",
+            "sample": f"{w.name}: whole replica ({rec1.L / 1e9:.2f} GB); "
+                      + ("JF64 over the committed /dev/shm image (every chunk, checked against the K1 digests); "
+                         if committed else f"JF64 on 1/{every} of the chunks (no /dev/shm image to read); ")
+                      + f"pack and unpack+verify on 1/{every} of the chunks, evenly spaced, extrapolated by bytes; "
+                      f"{nth} threads",
             "s_to_recover": full["s_to_recover"], "phases_s": full["phases_s"], "measured_s": full["measured_s"],
-            "coverage": {"layout": "full", "pack": f"sampled 1/{every}", "jf64": "full (committed image)",
+            "coverage": {"layout": "full", "pack": f"sampled 1/{every}",
+                         "jf64": "full (committed image)" if committed else f"sampled 1/{every}",
                          "select": "full", "shard": "full", "unpack_verify": f"sampled 1/{every}"},
             "digest_check": full["checks"],
             "single_thread": {"value": one["GBps"], "cores": 1, "s_to_recover": one["s_to_recover"],
@@ -473,7 +476,23 @@ def run_jitc(args):
         dist.broadcast_object_list(job, src=0)
     job = job[0]
     shm = args.image_dir or f"/dev/shm/jitc-bench-{job}"
-    if rank == 0 and not args.image_dir:   # also on an exception: never leave a 128 GB image behind
+    # N = 1 on a box whose /dev/shm cannot hold the image: private pinned host
+    # memory instead (jitc_config.image_dir = NULL, reading R16).
+    # N > 1 needs the shared image (every rank loads a slice of it).
+    image_kind = "shared /dev/shm"
+    if world == 1 and not args.image_dir:
+        need = sum(J.layout([(t.name, t.nbytes, 0) for t in g.tensors], 1 << 20)[2] for g in w.groups_of(rank))
+        try:
+            vfs = os.statvfs("/dev/shm")
+            free = vfs.f_bavail * vfs.f_frsize
+        except OSError:
+            free = 0
+        if args.private_image:
+            shm, image_kind = None, "private pinned (--private-image)"
+        elif free < need + (1 << 30):
+            shm, image_kind = None, f"private pinned (/dev/shm has {free / 1e9:.1f} GB free < {need / 1e9:.1f} GB)"
+            print(f"bench: {image_kind}", file=sys.stderr)
+    if rank == 0 and shm and not args.image_dir:   # also on an exception: never leave a 128 GB image behind
         import atexit
         atexit.register(lambda: [shutil.rmtree(d, ignore_errors=True) for d in (shm, f"{shm}-comm", f"{shm}-comm2")])
     flags = J.F_TIME_KERNELS
@@ -845,7 +864,7 @@ def run_jitc(args):
             "config": {"workload": w.name, "image_bytes": L_unique, "rank0_image_bytes": L_total,
                        "tensors": sum(len(g.tensors) for g in w.groups), "clip": args.clip or None,
                        "writers_k": {gs["group"]: len(gs["writers"]) for gs in sel_info["groups"]},
-                       "restore_mode": "HOST", "image": "shared /dev/shm",
+                       "restore_mode": "HOST", "image": image_kind,
                        "capture": "fanout" if fanout else "sharded", "victim": victim,
                        "transport": args.transport if world > 1 else None,
                        "comm_init_ms": round(comm_init_ms, 1) if world > 1 else None,
@@ -884,7 +903,8 @@ def run_jitc(args):
         if not args.no_cpu_baseline and world == 1:
             from oracle import oracle as O
             [(_, _, _, recs)] = O.decode_blobs(last_blob[0])
-            committed = {gid: np.memmap(f"{shm}/g{gid}.img", dtype=np.uint8, mode="r") for gid in states}
+            committed = ({gid: np.memmap(f"{shm}/g{gid}.img", dtype=np.uint8, mode="r") for gid in states}
+                         if shm else None)
             line["cpu_baseline"] = cpu_baseline(w, rank, last_blob[0], committed, {r.group: r.d for r in recs},
                                                 args.cpu_every, args.cpu_every_1t)
             del committed
@@ -892,7 +912,7 @@ def run_jitc(args):
     ctx.close()
     if world > 1:
         dist.barrier()
-    if rank == 0 and not args.image_dir:
+    if rank == 0 and shm and not args.image_dir:
         shutil.rmtree(shm, ignore_errors=True)
         shutil.rmtree(f"{shm}-comm", ignore_errors=True)
         shutil.rmtree(f"{shm}-comm2", ignore_errors=True)
@@ -917,6 +937,9 @@ def main():
                          "copy-engine transfer is amortised over 17 GB of K2/K3 traffic; DESIGN.md §7)")
     ap.add_argument("--zero-copy", action="store_true")
     ap.add_argument("--image-dir", default=None)
+    ap.add_argument("--private-image", action="store_true",
+                    help="N = 1: private pinned host image (image_dir = NULL) instead of /dev/shm; also chosen "
+                         "automatically when /dev/shm cannot hold the image")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-paper-protocol", action="store_true",
                     help="N > 1: skip the in-run comparison with the paper's every-rank-saves-everything protocol")
