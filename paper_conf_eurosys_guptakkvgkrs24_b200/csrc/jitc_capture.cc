@@ -7,8 +7,24 @@
 using namespace jitc;
 
 // ------------------------------------------------------------ capture (K2 + D2H)
-static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelection& gs, uint64_t v_star,
-                                 jitc_stats* stats) {
+// One pipeline over every group of the call: K2 packs round j of the writer's
+// shard into staging slot j % S on the compute stream, the copy stream D2Hs
+// it, and slot reuse is ordered by the ready/free events.  The round counter
+// runs on across groups, so a group's first K2 overlaps the previous group's
+// last D2H, and the call's first round is short (kFirstRound) so that the
+// copy engine starts within ~0.1 ms instead of after a whole 8 GiB K2
+// (pipeline fill).  Every group's re-digests are checked
+// against its fingerprint once the pipeline has drained.
+constexpr uint64_t kFirstRound = 512ull << 20;
+
+struct CapturePlan {
+  GroupState* g;
+  uint64_t c0, c1;
+};
+
+// Validation and the enqueue of one group's rounds; *j is the call's round counter.
+static jitc_status capture_enqueue(jitc_ctx* c, GroupState& g, const GroupSelection& gs, uint64_t v_star,
+                                   jitc_stats* stats, uint32_t* j, std::vector<CapturePlan>* todo) {
   if (gs.writers.empty()) {  // dropped OPTIONAL group: no checkpoint of it may survive
     drop_commit(c, g);
     return JITC_OK;
@@ -28,49 +44,57 @@ static jitc_status capture_group(jitc_ctx* c, GroupState& g, const GroupSelectio
   // byte (whichever writer starts first; unlink is idempotent)
   if (g.img_shm) unlink(gpath(c, g.id, ".commit").c_str());
   g.commit_priv.clear();
-  if (b1 > b0) {
-    CU(cudaMemsetAsync(g.d_dig2 + c0, 0, (c1 - c0) * 8, c->s_comp));
-    const bool zc = (c->cfg.flags & JITC_F_ZERO_COPY_D2H) != 0;
-    if (zc) {
-      uint32_t lo, hi;
-      seg_span(g, b0, b1, &lo, &hi);
-      jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, g.img_d, 0), g.d_dig2, b1 - b0);
-      if (st) return st;
-      if (stats) stats->rounds += 1, stats->d2h_bytes += b1 - b0;
-    } else {
-      const uint64_t R = c->slot_bytes;
-      const int nslots = (int)std::min<uint64_t>(jitc_ctx::kSlots, c->staging_bytes / R);
-      uint32_t j = 0;
-      for (uint64_t a = b0; a < b1; a += R, ++j) {
-        uint64_t b = std::min(a + R, b1);
-        int sl = (int)(j % nslots);
-        uint8_t* slot = c->staging + sl * R;
-        if (j >= (uint32_t)nslots) CU(cudaStreamWaitEvent(c->s_comp, c->ev_free[sl], 0));
-        c->tl_group = g.id, c->tl_round = j;
-        uint32_t lo, hi;
-        seg_span(g, a, b, &lo, &hi);
-        jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, slot, a), g.d_dig2, b - a);
-        if (st) return st;
-        CU(cudaEventRecord(c->ev_ready[sl], c->s_comp));
-        CU(cudaStreamWaitEvent(c->s_copy, c->ev_ready[sl], 0));
-        CU(copy_image(c, g, a, slot, b - a, cudaMemcpyDeviceToHost, c->s_copy));
-        CU(cudaEventRecord(c->ev_free[sl], c->s_copy));
-      }
-      if (stats) stats->rounds += j;
-      CU(cudaEventRecord(c->ev_join, c->s_copy));
-      CU(cudaStreamWaitEvent(c->s_comp, c->ev_join, 0));
-      if (stats) stats->d2h_bytes += b1 - b0;
-    }
-    CU(cudaMemcpyAsync(c->h_dig, g.d_dig2 + c0, (c1 - c0) * 8, cudaMemcpyDeviceToHost, c->s_comp));
+  g.captured = false;
+  todo->push_back({&g, c0, c1});
+  if (b1 <= b0) return JITC_OK;
+  CU(cudaMemsetAsync(g.d_dig2 + c0, 0, (c1 - c0) * 8, c->s_comp));
+  if (c->cfg.flags & JITC_F_ZERO_COPY_D2H) {
+    uint32_t lo, hi;
+    seg_span(g, b0, b1, &lo, &hi);
+    jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, g.img_d, 0), g.d_dig2, b1 - b0);
+    if (st) return st;
+    if (stats) stats->rounds += 1, stats->d2h_bytes += b1 - b0;
+    return JITC_OK;
   }
-  CU(cudaStreamSynchronize(c->s_comp));
-  for (uint64_t ch = c0; ch < c1; ++ch)
-    if (c->h_dig[ch - c0] != g.fp[ch])
+  const uint64_t R = c->slot_bytes;
+  const int nslots = (int)std::min<uint64_t>(jitc_ctx::kSlots, c->staging_bytes / R);
+  const uint64_t first = std::max<uint64_t>(g.C, std::min<uint64_t>(R, kFirstRound / g.C * g.C));
+  for (uint64_t a = b0; a < b1; ++*j) {
+    const uint64_t b = std::min(a + (*j == 0 ? first : R), b1);
+    const int sl = (int)(*j % nslots);
+    uint8_t* slot = c->staging + sl * R;
+    if (*j >= (uint32_t)nslots) CU(cudaStreamWaitEvent(c->s_comp, c->ev_free[sl], 0));
+    c->tl_group = g.id, c->tl_round = *j;
+    uint32_t lo, hi;
+    seg_span(g, a, b, &lo, &hi);
+    jitc_status st = run_segments(c, g, kPack, one_range(lo, hi, slot, a), g.d_dig2, b - a);
+    if (st) return st;
+    CU(cudaEventRecord(c->ev_ready[sl], c->s_comp));
+    CU(cudaStreamWaitEvent(c->s_copy, c->ev_ready[sl], 0));
+    CU(copy_image(c, g, a, slot, b - a, cudaMemcpyDeviceToHost, c->s_copy));
+    CU(cudaEventRecord(c->ev_free[sl], c->s_copy));
+    if (stats) stats->rounds += 1;
+    a = b;
+  }
+  if (stats) stats->d2h_bytes += b1 - b0;
+  return JITC_OK;
+}
+
+// After the pipeline drained: the re-digests of the writer's range must equal
+// its fingerprint (else the state changed between K1 and K2: EUNSTABLE).
+static jitc_status capture_check(jitc_ctx* c, const CapturePlan& p, uint64_t v_star, jitc_stats* stats) {
+  GroupState& g = *p.g;
+  if (p.c1 > p.c0) {
+    CU(cudaMemcpyAsync(c->h_dig, g.d_dig2 + p.c0, (p.c1 - p.c0) * 8, cudaMemcpyDeviceToHost, c->s_comp));
+    CU(cudaStreamSynchronize(c->s_comp));
+  }
+  for (uint64_t ch = p.c0; ch < p.c1; ++ch)
+    if (c->h_dig[ch - p.c0] != g.fp[ch])
       return fail(JITC_EUNSTABLE, "jitc_capture: group " + std::to_string(g.id) + " chunk " + std::to_string(ch) +
                                       " changed between fingerprint and capture");
   g.captured = true;
   g.cap_v = v_star;
-  if (stats) stats->image_bytes += b1 - b0;
+  if (stats) stats->image_bytes += std::min(p.c1 * g.C, g.L) - std::min(p.c0 * g.C, g.L);
   return JITC_OK;
 }
 
@@ -86,13 +110,35 @@ jitc_status jitc_capture(jitc_ctx* c, const void* selection, size_t sel_len, uin
   if (stats) memset(stats, 0, sizeof *stats), stats->first_bad_chunk = -1;
   CallTimer t(c);
   CU(cudaEventRecord(c->ev_t0, c->s_comp));
+  std::vector<CapturePlan> todo;
+  uint32_t j = 0;
+  jitc_status st = JITC_OK;
   for (auto& kv : c->groups) {
     GroupState& g = kv.second;
     if (!g.held || (group != JITC_ALL_GROUPS && g.id != group)) continue;
     const GroupSelection* gs = sel.find(g.id);
-    if (!gs) return fail(JITC_ELAYOUT, "jitc_capture: group missing from selection");
-    jitc_status st = capture_group(c, g, *gs, sel.v_star, stats);
-    if (st) return st;
+    if (!gs) {
+      st = fail(JITC_ELAYOUT, "jitc_capture: group missing from selection");
+      break;
+    }
+    st = capture_enqueue(c, g, *gs, sel.v_star, stats, &j, &todo);
+    if (st) break;
+  }
+  // drain the pipeline (also on an error: no copy may still read staging or
+  // write the image after the call returns)
+  CU(cudaEventRecord(c->ev_join, c->s_copy));
+  CU(cudaStreamWaitEvent(c->s_comp, c->ev_join, 0));
+  CU(cudaStreamSynchronize(c->s_comp));
+  if (st) {
+    harvest(c);
+    return st;
+  }
+  for (const CapturePlan& p : todo) {
+    st = capture_check(c, p, sel.v_star, stats);
+    if (st) {
+      harvest(c);
+      return st;
+    }
   }
   CU(cudaEventRecord(c->ev_t1, c->s_comp));
   CU(cudaEventSynchronize(c->ev_t1));

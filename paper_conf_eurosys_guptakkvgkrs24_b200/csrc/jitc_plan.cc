@@ -23,6 +23,9 @@
 
 namespace jitc {
 
+// HOST restore: length of the last round (see build_restore_plan).
+constexpr uint64_t kLastRound = 512ull << 20;
+
 static void o5_bytes(uint64_t n_c, uint64_t k, uint64_t s, uint64_t C, uint64_t L, uint64_t* a, uint64_t* b) {
   unsigned __int128 c0 = (unsigned __int128)s * n_c / k, c1 = (unsigned __int128)(s + 1) * n_c / k;
   *a = std::min<uint64_t>((uint64_t)c0 * C, L);
@@ -65,27 +68,46 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
       o5_bytes(n_c, n, r, C, L, &q0[r], &q1[r]);
       maxlen = std::max(maxlen, q1[r] - q0[r]);
     }
-    const uint64_t J = (maxlen + R - 1) / R;
+    // Round j covers bytes [off[j], off[j+1]) of every member's slice: R-byte
+    // rounds, except that the last one is short (kLastRound) so that the K3
+    // left after the last H2D is short (pipeline drain).  Block
+    // q of round j sits at base + q * len_j in the slot (len_j = the round's
+    // length, the all-gather's count).
+    // Boundaries are chunk multiples (a slice starts on a chunk and only the
+    // image's end is ragged), so no segment straddles two rounds.
+    std::vector<uint64_t> off{0};
+    const uint64_t last = std::max<uint64_t>(C, std::min<uint64_t>(R, kLastRound / C * C));
+    const uint64_t body = maxlen > last ? (maxlen - last + C - 1) / C * C : 0;
+    for (uint64_t x = 0; x < body; x = std::min(x + R, body)) off.push_back(std::min(x + R, body));
+    if (body < maxlen) off.push_back(maxlen);
+    const uint64_t J = off.size() - 1;
     *n_rounds = (uint32_t)J;
     for (uint64_t j = 0; j < J; ++j) {
       const uint32_t sl = (uint32_t)(j % S);
-      const uint64_t base = sl * n * R;
+      const uint64_t base = sl * n * R, len = off[j + 1] - off[j];
       const uint32_t rj = (uint32_t)j;
-      uint64_t a = q0[me] + j * R, b = std::min(q1[me], a + R);
-      if (b > a) ops->push_back(PlanOp{rj, kOpH2D, (uint8_t)sl, 0, in.me, 0, a, b, base + me * R, b - a});
+      auto range = [&](uint64_t q, uint64_t* a, uint64_t* b) {
+        *a = std::min(q1[q], q0[q] + off[j]);
+        *b = std::min(q1[q], q0[q] + off[j + 1]);
+      };
+      uint64_t a, b;
+      range(me, &a, &b);
+      if (b > a) ops->push_back(PlanOp{rj, kOpH2D, (uint8_t)sl, 0, in.me, 0, a, b, base + me * len, b - a});
       if (n > 1 && whole_comm) {
-        ops->push_back(PlanOp{rj, kOpAllGather, (uint8_t)sl, 0, -1, 0, 0, 0, base, R});
+        ops->push_back(PlanOp{rj, kOpAllGather, (uint8_t)sl, 0, -1, 0, 0, 0, base, len});
       } else if (n > 1) {
         for (uint64_t q = 0; q < n; ++q) {
           if (q == me) continue;
-          if (b > a) ops->push_back(PlanOp{rj, kOpSend, (uint8_t)sl, 0, P[q], 0, a, b, base + me * R, b - a});
-          uint64_t qa = q0[q] + j * R, qb = std::min(q1[q], qa + R);
-          if (qb > qa) ops->push_back(PlanOp{rj, kOpRecv, (uint8_t)sl, 0, P[q], 0, qa, qb, base + q * R, qb - qa});
+          if (b > a) ops->push_back(PlanOp{rj, kOpSend, (uint8_t)sl, 0, P[q], 0, a, b, base + me * len, b - a});
+          uint64_t qa, qb;
+          range(q, &qa, &qb);
+          if (qb > qa) ops->push_back(PlanOp{rj, kOpRecv, (uint8_t)sl, 0, P[q], 0, qa, qb, base + q * len, qb - qa});
         }
       }
       for (uint64_t q = 0; q < n; ++q) {
-        uint64_t qa = q0[q] + j * R, qb = std::min(q1[q], qa + R);
-        if (qb > qa) ops->push_back(PlanOp{rj, kOpUnpack, (uint8_t)sl, 0, P[q], 0, qa, qb, base + q * R, qb - qa});
+        uint64_t qa, qb;
+        range(q, &qa, &qb);
+        if (qb > qa) ops->push_back(PlanOp{rj, kOpUnpack, (uint8_t)sl, 0, P[q], 0, qa, qb, base + q * len, qb - qa});
       }
     }
     return true;
