@@ -23,8 +23,22 @@
 
 namespace jitc {
 
-// HOST restore: length of the last round (see build_restore_plan).
+// Round boundaries [off[j], off[j+1]) within every participant's range of
+// at most maxlen bytes: R-byte rounds, except that the last one is short
+// (kLastRound, capped at R) so that the K3 left after the last transfer is
+// short (pipeline drain).  Boundaries are chunk multiples (a
+// range starts on a chunk and only the image's end is ragged), so no segment
+// straddles two rounds.
 constexpr uint64_t kLastRound = 512ull << 20;
+
+static std::vector<uint64_t> round_offsets(uint64_t maxlen, uint64_t R, uint64_t C) {
+  std::vector<uint64_t> off{0};
+  const uint64_t last = std::max<uint64_t>(C, std::min<uint64_t>(R, kLastRound / C * C));
+  const uint64_t body = maxlen > last ? (maxlen - last + C - 1) / C * C : 0;
+  for (uint64_t x = 0; x < body; x = std::min(x + R, body)) off.push_back(std::min(x + R, body));
+  if (body < maxlen) off.push_back(maxlen);
+  return off;
+}
 
 static void o5_bytes(uint64_t n_c, uint64_t k, uint64_t s, uint64_t C, uint64_t L, uint64_t* a, uint64_t* b) {
   unsigned __int128 c0 = (unsigned __int128)s * n_c / k, c1 = (unsigned __int128)(s + 1) * n_c / k;
@@ -68,18 +82,10 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
       o5_bytes(n_c, n, r, C, L, &q0[r], &q1[r]);
       maxlen = std::max(maxlen, q1[r] - q0[r]);
     }
-    // Round j covers bytes [off[j], off[j+1]) of every member's slice: R-byte
-    // rounds, except that the last one is short (kLastRound) so that the K3
-    // left after the last H2D is short (pipeline drain).  Block
+    // Round j covers bytes [off[j], off[j+1]) of every member's slice.  Block
     // q of round j sits at base + q * len_j in the slot (len_j = the round's
     // length, the all-gather's count).
-    // Boundaries are chunk multiples (a slice starts on a chunk and only the
-    // image's end is ragged), so no segment straddles two rounds.
-    std::vector<uint64_t> off{0};
-    const uint64_t last = std::max<uint64_t>(C, std::min<uint64_t>(R, kLastRound / C * C));
-    const uint64_t body = maxlen > last ? (maxlen - last + C - 1) / C * C : 0;
-    for (uint64_t x = 0; x < body; x = std::min(x + R, body)) off.push_back(std::min(x + R, body));
-    if (body < maxlen) off.push_back(maxlen);
+    const std::vector<uint64_t> off = round_offsets(maxlen, R, C);
     const uint64_t J = off.size() - 1;
     *n_rounds = (uint32_t)J;
     for (uint64_t j = 0; j < J; ++j) {
@@ -146,24 +152,33 @@ bool build_restore_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
     o5_bytes(n_c, k, s, C, L, &q0[s], &q1[s]);
     maxlen = std::max(maxlen, q1[s] - q0[s]);
   }
-  const uint64_t J = (maxlen + R - 1) / R;
+  // round j covers bytes [off[j], off[j+1]) of every writer's range
+  const std::vector<uint64_t> roff = round_offsets(maxlen, R, C);
+  const uint64_t J = roff.size() - 1;
   *n_rounds = (uint32_t)J;
+  auto range = [&](uint64_t s, uint64_t j, uint64_t* a, uint64_t* b) {
+    *a = std::min(q1[s], q0[s] + roff[j]);
+    *b = std::min(q1[s], q0[s] + roff[j + 1]);
+  };
   for (uint64_t j = 0; j < J; ++j) {
     const uint32_t sl = (uint32_t)(j % S);
     const uint64_t base = sl * k * R;   // block s of a round sits at base + s*R on every rank
     if (my_s >= 0) {
-      uint64_t a = q0[my_s] + j * R, b = std::min(q1[my_s], a + R);
+      uint64_t a, b;
+      range((uint64_t)my_s, j, &a, &b);
       if (b <= a) continue;
       const uint64_t off = base + (uint64_t)my_s * R;
       ops->push_back(PlanOp{(uint32_t)j, kOpPack, (uint8_t)sl, 0, in.me, 0, a, b, off, b - a});
       for (int32_t d : in.dests) ops->push_back(PlanOp{(uint32_t)j, kOpSend, (uint8_t)sl, 0, d, 0, a, b, off, b - a});
     } else {
       for (uint64_t s = 0; s < k; ++s) {
-        uint64_t a = q0[s] + j * R, b = std::min(q1[s], a + R);
+        uint64_t a, b;
+        range(s, j, &a, &b);
         if (b > a) ops->push_back(PlanOp{(uint32_t)j, kOpRecv, (uint8_t)sl, 0, in.writers[s], 0, a, b, base + s * R, b - a});
       }
       for (uint64_t s = 0; s < k; ++s) {
-        uint64_t a = q0[s] + j * R, b = std::min(q1[s], a + R);
+        uint64_t a, b;
+        range(s, j, &a, &b);
         if (b > a) ops->push_back(PlanOp{(uint32_t)j, kOpUnpack, (uint8_t)sl, 0, in.writers[s], 0, a, b, base + s * R, b - a});
       }
     }
