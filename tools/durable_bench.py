@@ -20,6 +20,54 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
+def raw_disk(dirpath: str, nbytes: int, threads: int = 8, piece: int = 64 << 20) -> dict:
+    """The disk's own rate for the library's access pattern (the NEXT-4
+    roofline): `threads` threads pwrite / pread 64 MiB pieces of one file with
+    O_DIRECT, fdatasync after the writes, page cache dropped before the reads."""
+    import mmap
+    import threading
+    path = os.path.join(dirpath, "raw-baseline.bin")
+    buf = mmap.mmap(-1, piece)                      # page-aligned, as O_DIRECT needs
+    buf.write(os.urandom(1 << 20) * (piece >> 20))
+
+    def run(write: bool) -> float:
+        flags = (os.O_WRONLY | os.O_CREAT | os.O_TRUNC) if write else os.O_RDONLY
+        fd = os.open(path, flags | getattr(os, "O_DIRECT", 0), 0o600)
+        if write:
+            os.ftruncate(fd, nbytes)
+        mv = memoryview(buf)
+
+        def work(t):
+            for off in range(t * piece, nbytes, threads * piece):
+                n = min(piece, nbytes - off)
+                if write:
+                    os.pwrite(fd, mv[:n], off)
+                else:
+                    os.preadv(fd, [mv[:n]], off)
+        t0 = time.perf_counter()
+        ths = [threading.Thread(target=work, args=(t,)) for t in range(threads)]
+        for th in ths:
+            th.start()
+        for th in ths:
+            th.join()
+        if write:
+            os.fdatasync(fd)
+        dt = time.perf_counter() - t0
+        os.close(fd)
+        return nbytes / dt / 1e9
+    w = run(True)
+    subprocess.run(["sync"])
+    try:
+        with open("/proc/sys/vm/drop_caches", "w") as f:
+            f.write("1\n")
+    except OSError:
+        pass
+    r = run(False)
+    os.unlink(path)
+    return {"bytes": nbytes, "threads": threads, "piece_MiB": piece >> 20, "write_GBps": round(w, 3),
+            "read_GBps": round(r, 3), "how": "O_DIRECT pwrite/pread of 64 MiB pieces, fdatasync, cache dropped"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="C2")
@@ -72,6 +120,10 @@ def main():
                "stage_in_s": round(t_s, 3), "stage_in_GBps": round(q["image_bytes"] / t_s / 1e9, 3),
                "page_cache_dropped_before_stage_in": cold,
                "restore_after_stage_in": "bit-exact (every chunk digest == manifest; verify == fingerprint)"}
+        raw = raw_disk(args.dir, min(g.nbytes, 16 << 30), threads=int(os.environ.get("JITC_DURABLE_THREADS", 8)))
+        out["raw_disk"] = raw
+        out["persist_frac_of_raw_write"] = round(out["persist_GBps"] / raw["write_GBps"], 3)
+        out["stage_in_frac_of_raw_read"] = round(out["stage_in_GBps"] / raw["read_GBps"], 3)
         print(json.dumps(out), flush=True)
     finally:
         ctx.close()
