@@ -135,6 +135,10 @@ def calibrate_links(device: int, world: int, nccl_group=None, host_gib: int = 2)
     a = torch.empty(4 << 30, dtype=torch.uint8, device=f"cuda:{device}")
     b = torch.empty_like(a)
     out["hbm_copy_GBps"] = round(2 * a.numel() / timed(lambda: b.copy_(a)) / 1e9, 1)
+    # read-only reference for K1 (which only reads): torch's int64 sum over the
+    # same 4 GiB (a reduction with a negligible write)
+    a.zero_()
+    out["hbm_read_GBps"] = round(a.numel() / timed(lambda: a.view(torch.int64).sum()) / 1e9, 1)
     del a, b, d
     if nccl_group is not None and world > 1:
         blk = torch.empty(256 << 20, dtype=torch.uint8, device=f"cuda:{device}")
@@ -143,7 +147,7 @@ def calibrate_links(device: int, world: int, nccl_group=None, host_gib: int = 2)
         out["nvl_allgather_busbw_GBps"] = round((world - 1) * blk.numel() / t / 1e9, 1)
     torch.cuda.empty_cache()
     out["how"] = (f"{host_gib} GiB pinned, 64 MiB pieces, all {world} rank(s) at once, best of 5, after the warm-up steps; "
-                  "HBM: 4 GiB D2D copy (read+write)")
+                  "HBM: 4 GiB D2D copy (read+write); HBM read: torch int64 sum over the 4 GiB")
     return out
 
 
@@ -811,6 +815,8 @@ def run_jitc(args):
                                                      "achieved": round(local / (ms * 1e-3) / 1e9, 1),
                                                      "frac": round(local / (ms * 1e-3) / 1e9 / peak, 4)}}
         out["bound"] = "hbm"
+        if k == J.K_DIGEST and links and links.get("hbm_read_GBps"):   # K1 only reads: also vs a read-only rate
+            out["hbm"]["frac_of_read_calibration"] = round(local / (ms * 1e-3) / 1e9 / links["hbm_read_GBps"], 4)
         if remote:
             out["nvlink"] = {"bytes_per_launch": remote, "achieved": round(remote / (ms * 1e-3) / 1e9, 1),
                              "frac": round(remote / (ms * 1e-3) / 1e9 / nvl_peak, 4)}
