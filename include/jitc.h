@@ -239,8 +239,12 @@ jitc_status jitc_select_consistent_replica(const void* blobs, size_t len, const 
  * [floor(s*n_c/k), floor((s+1)*n_c/k)) (O5) into the host image, in rounds:
  * K2 gathers the tensors into a staging slot (or straight into mapped host
  * memory with JITC_F_ZERO_COPY_D2H) re-digesting every chunk, and the copy
- * stream drains the slot D2H while K2 fills the next.  A re-digest that
- * differs from the last jitc_fingerprint => JITC_EUNSTABLE.  A non-writer
+ * stream drains the slot D2H while K2 fills the next.  The rounds of all
+ * groups of the call form one pipeline whose first round is 512 MiB (so the
+ * copy engine starts at once).  A re-digest that differs from the last
+ * jitc_fingerprint => JITC_EUNSTABLE (checked after the pipeline drained;
+ * the group then counts as not captured, so jitc_commit refuses it).  On any
+ * error the call returns only after its copies finished.  A non-writer
  * returns JITC_OK having done nothing, so every rank can call it. */
 jitc_status jitc_capture(jitc_ctx* ctx, const void* selection, size_t sel_len, uint32_t group,
                          jitc_stats* stats);
@@ -365,7 +369,9 @@ jitc_status jitc_persist(jitc_ctx* ctx, uint32_t group, const char* dir, jitc_st
 /* Reads a durable copy back into the host image (validating the commit
  * record, the manifest trailer and the layout: JITC_EINCOMPLETE /
  * JITC_ELAYOUT) and installs its manifest, so that jitc_restore(HOST)
- * restores it with full K3 verification. */
+ * restores it with full K3 verification.  O_DIRECT reads go through two
+ * 64 MiB bounce buffers per I/O thread (8 threads; JITC_DURABLE_THREADS),
+ * the copy into the image overlapping the next read. */
 jitc_status jitc_stage_in(jitc_ctx* ctx, uint32_t group, const char* dir, jitc_stats* stats);
 
 /* ---- hang detection (NEXT-1; §3.1-3.2) ------------------ */
