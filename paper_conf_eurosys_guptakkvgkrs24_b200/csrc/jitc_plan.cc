@@ -241,17 +241,32 @@ bool build_capture_plan(const PlanInput& in, std::vector<PlanOp>* ops, uint64_t*
     uint64_t a, b;
     uint32_t q;
   };
+  // Writer s cuts the part of its shard in each lane into <= R blocks and
+  // visits the lanes round-robin (lane q's i-th block, then lane q+1's i-th
+  // block, ...), so consecutive rounds go to different movers and every
+  // mover's D2H runs at once.  Lane-major order (all of lane q's blocks,
+  // then lane q+1's) would keep one or two movers busy at a time: a mover's
+  // slot is reused two rounds later and its D2H takes far longer than the
+  // K2 + NVLink transfer that feed it (tools/fanout_sim.py).
   std::vector<std::vector<Block>> blocks(k);
   uint64_t J = 0;
   for (uint64_t s = 0; s < k; ++s) {
     uint64_t a, b;
     o5_bytes(n_c, k, s, C, L, &a, &b);
+    std::vector<std::vector<Block>> per_lane;
+    size_t most = 0;
     for (uint64_t q = 0; q < m; ++q) {
       uint64_t la, lb;
       o5_bytes(n_c, m, q, C, L, &la, &lb);
       const uint64_t x = std::max(a, la), y = std::min(b, lb);
-      for (uint64_t u = x; u < y; u += R) blocks[s].push_back(Block{u, std::min(u + R, y), (uint32_t)q});
+      if (x >= y) continue;
+      per_lane.emplace_back();
+      for (uint64_t u = x; u < y; u += R) per_lane.back().push_back(Block{u, std::min(u + R, y), (uint32_t)q});
+      most = std::max(most, per_lane.back().size());
     }
+    for (size_t i = 0; i < most; ++i)
+      for (auto& lane : per_lane)
+        if (i < lane.size()) blocks[s].push_back(lane[i]);
     J = std::max<uint64_t>(J, blocks[s].size());
   }
   *n_rounds = (uint32_t)J;

@@ -186,3 +186,38 @@ def test_plan_errors(J, group):
         J.capture_plan(sel, 0, [0, 1], [0, 1], 0, C, C)                 # staging below 2 * k * C
     with pytest.raises(J.JitcError):
         J.capture_plan(sel, 9, [0, 1], [0, 1], 0, 1 << 20, 1 << 18)    # group not in the selection
+
+
+def test_round_robin_lanes_match_timing_model(J, group):
+    """The library's fan-out plan visits the movers' lanes round-robin (each
+    writer's j-th block goes to the next lane it intersects), exactly as
+    tools/fanout_sim.py models it -- so that model's projections (DESIGN.md
+    §8.6) describe the executed schedule -- and consecutive rounds of a lone
+    writer go to different movers."""
+    import importlib.util
+    import os
+    spec = importlib.util.spec_from_file_location(
+        "fanout_sim", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools", "fanout_sim.py"))
+    sim = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(sim)
+    sim.C = C
+    lay, img = group
+    for topo, healthy, gid, movers in (({0: [0, 1]}, [0], 0, [0, 1]),
+                                       ({0: [0, 1, 2, 3]}, [0, 1], 0, [0, 1, 2, 3]),
+                                       ({0: [0, 2], 1: [1, 3]}, [0, 1, 2], 1, [0, 1, 2])):
+        sel = _selection(J, lay, img, topo, healthy)
+        gs = next(g for g in J.parse_selection(sel)["groups"] if g["group"] == gid)
+        writers = gs["writers"]
+        for staging, slot in ((8 * C * 4, 4 * C), (6 * C * 4, 3 * C), (4 * C, C)):
+            if staging < 2 * len(writers) * C:
+                continue
+            R = min(slot, staging // (2 * len(writers))) // C * C
+            want = sim.blocks_of(lay.n_c, lay.L, len(writers), len(movers), R, "round-robin")
+            for s, w in enumerate(writers):
+                plan = J.capture_plan(sel, gid, movers, list(range(4)), w, staging, slot)
+                packs = [(op["round"], op["a"], op["b"]) for op in plan["ops"] if op["kind"] == "PACK"]
+                assert packs == [(j, a, b) for j, (a, b, q) in enumerate(want[s])]
+            if len(writers) == 1:
+                lanes = [q for a, b, q in want[0]]
+                n_lanes = len(set(lanes))
+                assert all(x != y for x, y in zip(lanes, lanes[1:])) or n_lanes == 1
