@@ -352,12 +352,27 @@ static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::strin
     work();
     for (auto& th : pool) th.join();
   };
-  // 1. allocate the pages and fill this process's page tables, in parallel;
-  //    kernels without MADV_POPULATE_WRITE (< 5.14) fall back to fallocate
+  // 1. allocate the pages and fill this process's page tables, in parallel,
+  //    and pin each piece right after populating it (page zeroing and the
+  //    driver's pinning overlap across the pool: C3 setup 23 s on average
+  //    against 33 s populating everything first, tools/setup_probe.py,
+  //    profiles/r02f_setup_probe.txt; JITC_PIN_FUSED=0 restores the two
+  //    phases).  Kernels without MADV_POPULATE_WRITE (< 5.14) fall back to
+  //    fallocate and pin afterwards.
   std::atomic<int> pop_err{0};
+  const bool fused = !(getenv("JITC_PIN_FUSED") && atoi(getenv("JITC_PIN_FUSED")) == 0);
+  std::vector<cudaError_t> rc(n_pieces, cudaSuccess);
+  std::vector<char> pinned(n_pieces, 0);
   pool_run([&](uint64_t i) {
     const uint64_t a = i * piece, n = std::min(piece, g.img_bytes - a);
-    if (madvise(static_cast<uint8_t*>(p) + a, n, 23 /* MADV_POPULATE_WRITE */) != 0) pop_err = errno;
+    if (madvise(static_cast<uint8_t*>(p) + a, n, 23 /* MADV_POPULATE_WRITE */) != 0) {
+      pop_err = errno;
+      return;
+    }
+    if (fused) {
+      rc[i] = cudaHostRegister(static_cast<uint8_t*>(p) + a, n, cudaHostRegisterMapped | cudaHostRegisterPortable);
+      pinned[i] = 1;
+    }
   });
   if (pop_err) {
     const int e = pop_err == EINVAL ? posix_fallocate(fd, 0, (off_t)g.img_bytes) : (int)pop_err;
@@ -369,12 +384,12 @@ static jitc_status map_shared_image(jitc_ctx* c, GroupState& g, const std::strin
   }
   close(fd);
   const double t_populated = now_ms();
-  // 2. pin the populated pieces (no fresh page is faulted in by the driver,
+  // 2. pin what step 1 did not (no fresh page is faulted in by the driver,
   //    so ranks of a box may register the same image concurrently)
-  std::vector<cudaError_t> rc(n_pieces, cudaSuccess);
   pool_run([&](uint64_t i) {
     const uint64_t a = i * piece, n = std::min(piece, g.img_bytes - a);
-    rc[i] = cudaHostRegister(static_cast<uint8_t*>(p) + a, n, cudaHostRegisterMapped | cudaHostRegisterPortable);
+    if (!pinned[i])
+      rc[i] = cudaHostRegister(static_cast<uint8_t*>(p) + a, n, cudaHostRegisterMapped | cudaHostRegisterPortable);
   });
   if (getenv("JITC_DEBUG_TIMING"))
     fprintf(stderr,
