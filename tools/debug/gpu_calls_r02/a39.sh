@@ -1,0 +1,6 @@
+# call 39 (settle only judges captures >= 4 GiB per rank): bench with the bounded settle loop (C2 N=1, and a 2-rank dry run)
+mkdir -p gpurun_out
+timeout 900 python bench.py --config C2 --steps 3 --no-cpu-baseline > gpurun_out/a39_c2.json 2> gpurun_out/a39_c2.err; echo EXIT=$? >> gpurun_out/a39_c2.err
+JITC_BENCH_SHARE_GPU=1 timeout 900 python -m torch.distributed.run --nnodes=1 --master-addr 127.0.0.1 --nproc-per-node 2 --master-port 29582 bench.py --gpus 2 --config C1 --steps 3 --warmup 3 \
+  --no-cpu-baseline --staging 512 --slot 128 > gpurun_out/a39_c1_n2.json 2> gpurun_out/a39_c1_n2.err; echo EXIT=$? >> gpurun_out/a39_c1_n2.err
+echo done
