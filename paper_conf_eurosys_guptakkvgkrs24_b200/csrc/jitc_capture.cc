@@ -388,6 +388,16 @@ static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelec
 // The local part of jitc_commit: manifest + commit record of every group this
 // rank is the lowest writer of; dropped groups lose any older checkpoint.
 static jitc_status commit_groups(jitc_ctx* c, const Selection& sel) {
+  // every group this rank writes must be captured at v* before any manifest
+  // or commit record is written (no partial commit of a multi-group call)
+  for (auto& kv : c->groups) {
+    const GroupState& g = kv.second;
+    const GroupSelection* gs = g.held ? sel.find(g.id) : nullptr;
+    if (!gs || gs->writers.empty()) continue;
+    if (std::find(gs->writers.begin(), gs->writers.end(), c->cfg.rank) == gs->writers.end()) continue;
+    if (!g.captured || g.cap_v != sel.v_star)
+      return fail(JITC_ESTATE, "jitc_commit: group " + std::to_string(g.id) + " not captured at v*");
+  }
   for (auto& kv : c->groups) {
     GroupState& g = kv.second;
     if (!g.held) continue;

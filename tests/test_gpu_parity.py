@@ -365,6 +365,48 @@ def test_unstable_between_fingerprint_and_capture(J, shm):
     assert e.value.status == J.EUNSTABLE
 
 
+def test_capture_pipeline_across_groups(J, shm):
+    """jitc_capture runs the rounds of all groups as one pipeline (short first
+    round, slots carried across groups): every group's image == the oracle's
+    pack; a change in the SECOND group between fingerprint and capture is
+    EUNSTABLE naming that group, after which commit refuses before writing
+    anything (the group is not captured; no group gets a commit record) and a
+    fresh fingerprint -> capture -> commit -> restore works."""
+    C = 4096
+    gs = [W.random_table(40 + i, 50, max_bytes=30000, group=i) for i in range(3)]
+    sts = [_state(g, 8 + g.group) for g in gs]
+    ctx = _ctx(J, C, image_dir=shm, staging=8 * C * 4, slot=4 * C)   # rounds of 4 chunks, 8 slots
+    for g, st in zip(gs, sts):
+        ctx.register(g.group, J.REQUIRED, [0], st.table(), keepalive=st)
+        ctx.mark(g.group, 4, J.CLEAN)
+    blob = ctx.fingerprint()
+    st_, sel = J.select_consistent_replica(blob, [0])
+    J.inject_bitflip(sts[1].ptrs[3], 0, 1)
+    with pytest.raises(J.JitcError) as e:
+        ctx.capture(sel)
+    assert e.value.status == J.EUNSTABLE and "group 1" in str(e.value)
+    with pytest.raises(J.JitcError) as e:
+        ctx.commit(sel)
+    assert e.value.status == J.ESTATE
+    assert not any(os.path.exists(f"{shm}/g{g.group}.commit") for g in gs), "no partial commit"
+    J.inject_bitflip(sts[1].ptrs[3], 0, 1)                    # undo: the state is the oracle's again
+    blob, sel, cap = _pipeline(J, ctx)
+    assert cap["rounds"] >= 3
+    for g in gs:
+        lay = O.layout_of_group(g, C)
+        img = np.fromfile(f"{shm}/g{g.group}.img", dtype=np.uint8)[:lay.L]
+        assert np.array_equal(img, O.pack(O.gen_group(g, 8 + g.group), lay)), g.group
+    for st in sts:
+        st.scramble()
+    ctx.restore(J.ALL_GROUPS, J.HOST)
+    torch.cuda.synchronize()
+    for g, st in zip(gs, sts):
+        for i, t in enumerate(g.tensors):
+            assert np.array_equal(st.tensor_bytes(i).cpu().numpy(), O.gen_tensor_bytes(t, 8 + g.group, g.group))
+        assert ctx.verify(g.group, blob) == 2**64 - 1
+    ctx.close()
+
+
 def test_half_step_detected(J):
     """A half-applied optimizer step (U_v on tensors [0, split)) changes exactly
     the chunks the oracle predicts, and the replica class splits."""
