@@ -387,9 +387,10 @@ static std::vector<uint8_t> build_manifest(const GroupState& g, const GroupSelec
 
 // The local part of jitc_commit: manifest + commit record of every group this
 // rank is the lowest writer of; dropped groups lose any older checkpoint.
-static jitc_status commit_groups(jitc_ctx* c, const Selection& sel) {
-  // every group this rank writes must be captured at v* before any manifest
-  // or commit record is written (no partial commit of a multi-group call)
+// Every group this rank writes must be captured at v* before any manifest or
+// commit record is written anywhere (the ranks agree on it first), so a
+// multi-group commit is all or nothing.
+static jitc_status commit_check(jitc_ctx* c, const Selection& sel) {
   for (auto& kv : c->groups) {
     const GroupState& g = kv.second;
     const GroupSelection* gs = g.held ? sel.find(g.id) : nullptr;
@@ -398,6 +399,10 @@ static jitc_status commit_groups(jitc_ctx* c, const Selection& sel) {
     if (!g.captured || g.cap_v != sel.v_star)
       return fail(JITC_ESTATE, "jitc_commit: group " + std::to_string(g.id) + " not captured at v*");
   }
+  return JITC_OK;
+}
+
+static jitc_status commit_groups(jitc_ctx* c, const Selection& sel) {
   for (auto& kv : c->groups) {
     GroupState& g = kv.second;
     if (!g.held) continue;
@@ -443,6 +448,9 @@ jitc_status jitc::commit_impl(jitc_ctx* c, const void* selection, size_t sel_len
   if (sel.status != JITC_OK) return fail(sel.status, "jitc_commit: selection status is not OK");
   CU(cudaSetDevice(c->device));
   jitc_status st = collective ? barrier(c) : JITC_OK;  // every writer's capture has returned
+  if (st) return st;
+  st = commit_check(c, sel);
+  if (collective && has_comm(c)) st = agree(c, st);    // nobody writes unless every writer can
   if (st) return st;
   st = commit_groups(c, sel);
   // nobody restores before every commit record exists, and a rank that failed
