@@ -399,7 +399,12 @@ cudaError_t preload_kernels() {
     cudaError_t e = cudaFuncGetAttributes(&fa, f);
     if (e != cudaSuccess) return e;
   }
-  return cudaSuccess;
+  // the grid sizes too, so that no launch in the failure path queries the device
+  per_sm<kDigest>();
+  per_sm<kPack>();
+  per_sm<kUnpack>();
+  per_sm<kPull>();
+  return cudaGetLastError();
 }
 
 cudaError_t device_check(int device, std::string* why) {
