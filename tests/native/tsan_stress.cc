@@ -3,7 +3,7 @@
 // Runs every thread the library starts -- the IPC heartbeat thread, the
 // liveness heartbeat thread (jitc_liveness_init), the watchdog thread and its
 // on-hang capture action (local and collective), the parallel pinning pool of
-// jitc_register -- while other threads make the calls the header allows
+// jitc_register, the durable tier's I/O and copier threads -- while other threads make the calls the header allows
 // during a watchdog (jitc_watch_event, jitc_watchdog_wait, jitc_watchdog_failed,
 // jitc_watchdog_stop).  Built with -fsanitize=thread (the runtime lives in
 // this executable); the library's host code is instrumented too.  Prints
@@ -134,6 +134,16 @@ int main(int argc, char** argv) {
       return 4;
     }
     fired_total += fired;
+  }
+  // the durable tier's I/O threads and stage-in's bounce-buffer copier threads
+  // (argv[3]: a directory on a disk file system, so that O_DIRECT is used)
+  if (argc > 3) {
+    jitc_stats ds;
+    CHECK(jitc_persist(c, 0, argv[3], &ds));
+    CHECK(jitc_stage_in(c, 0, argv[3], &ds));
+    CHECK(jitc_restore(c, 0, JITC_RESTORE_HOST, nullptr, 0, &ds));
+    uint64_t bad = 0;
+    CHECK(jitc_verify(c, 0, nullptr, 0, &bad));
   }
   int32_t dead[4], nd = 0;
   CHECK(jitc_comm_dead(c, dead, 4, &nd));

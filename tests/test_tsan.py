@@ -51,10 +51,12 @@ def test_threads_under_tsan():
         # unlocked mutex in ld-linux, measured on B200)
         f.write("called_from_lib:libcuda.so\nmutex:ld-linux-x86-64.so.2\nmutex:libnccl.so.2\n")
     env = dict(os.environ, TSAN_OPTIONS=f"halt_on_error=1 second_deadlock_stack=1 suppressions={supp}")
+    durable = f"/tmp/jitc-tsan-durable-{os.getpid()}-{uuid.uuid4().hex[:8]}"   # a disk file system: O_DIRECT
     try:
-        r = subprocess.run([exe, d, "6"], env=env, capture_output=True, text=True, timeout=600)
+        r = subprocess.run([exe, d, "6", durable], env=env, capture_output=True, text=True, timeout=600)
     finally:
         shutil.rmtree(d, ignore_errors=True)
+        shutil.rmtree(durable, ignore_errors=True)
     out = r.stdout + r.stderr
     assert "ThreadSanitizer" not in out, out[-6000:]
     assert r.returncode == 0 and "tsan-ok" in r.stdout, out[-4000:]
